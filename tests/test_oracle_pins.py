@@ -1,0 +1,292 @@
+"""Pins of the CPU oracle against the paper and the mathematics (no GPU).
+
+Each test names what it pins.
+None of these retypes an oracle formula: they compare it with values the paper
+prints for its worked examples, closed forms, an independent library routine
+(numpy lexsort) on tiny inputs, brute force, the paper's quality theorem, and
+invariants that any correct implementation satisfies.
+"""
+import itertools
+
+import numpy as np
+import pytest
+
+import oracle
+import ganns_synth as syn
+
+
+# ----------------------------------------------------------------- O1 (R-C9)
+def test_distance_closed_forms():
+    # hand-computed: (1-4)^2 + (2-6)^2 = 25
+    assert oracle.distance([1, 2, 3, 4], [4, 6, 3, 4], "l2") == 25.0
+    # -<(1,2,3,4),(2,0,-1,1)> = -(2 + 0 - 3 + 4) = -3
+    assert oracle.distance([1, 2, 3, 4], [2, 0, -1, 1], "ip") == -3.0
+    # 1 - <(3,4,0,0),(1,0,0,0)> / 5 = 0.4
+    assert abs(oracle.distance([3, 4, 0, 0], [1, 0, 0, 0], "cosine") - 0.4) < 1e-7
+    # orthogonal IP is +0.0, never -0.0 (total order on keys)
+    z = oracle.distance([1, 0, 0, 0], [0, 1, 0, 0], "ip")
+    assert z == 0.0 and np.signbit(np.float32(z)) == False  # noqa: E712
+
+
+def test_distance_matches_numpy_float64():
+    rng = np.random.default_rng(1)
+    for metric in ("l2", "ip", "cosine"):
+        for d in (4, 8, 128, 960):
+            q = rng.standard_normal(d).astype(np.float32)
+            x = rng.standard_normal(d).astype(np.float32)
+            q64, x64 = q.astype(np.float64), x.astype(np.float64)
+            ref = {"l2": ((q64 - x64) ** 2).sum(), "ip": -(q64 @ x64),
+                   "cosine": 1 - (q64 @ x64) / np.linalg.norm(q64)}[metric]
+            assert oracle.distance(q, x, metric) == np.float32(ref)
+
+
+# ----------------------------------------------------------- P1: Example 2
+def test_example2_trace(g1):
+    """GANNS on Fig. 1: T of iteration 1 sorts v8,v7,v2,v5,v3; path
+    v1->v8->v10->v12->v9; iteration 5 explores v9 (the only unexplored point) and
+    leaves N unchanged; returns v12, v9, v8, v10."""
+    ex = g1["ex2"]
+    tr = oracle.search_trace(g1["nbr"], g1["X"], g1["q"], k=4, l=4, e=4, entry=0)
+    assert tr["explored"].tolist() == [it["explore"] for it in ex["its"]]
+    for i, it in enumerate(ex["its"]):
+        assert tr["N"][i].tolist() == it["N"], f"iteration {i + 1}"
+        assert tr["flags"][i].tolist() == it["flags"], f"iteration {i + 1}"
+        t = tr["T"][i]
+        assert t[t >= 0].tolist() == it["tsorted"], f"iteration {i + 1}"
+    assert tr["ids"].tolist() == ex["result"]
+    assert tr["dists"].tolist() == ex["dists"]
+    assert tr["stats"].tolist() == ex["stats"]
+    # iteration 5 leaves N unchanged
+    assert tr["N"][4].tolist() == tr["N"][3].tolist()
+
+
+def test_example2_literal_dup_reading_is_rejected(g1):
+    """R-C1: the oracle drops duplicates; its result equals the paper's list.  The
+    alternative reading ("keep duplicates, flag them explored") would return v12
+    twice -- a contradiction with P:214 -- so the oracle must never emit a repeated id."""
+    ids, _ = oracle.search(g1["nbr"], g1["X"], g1["q"][None], k=4, l=4)
+    assert len(set(ids[0].tolist())) == 4
+
+
+# ----------------------------------------------------------- P2: Example 1
+def test_example1_trace(g1):
+    """Algorithm 1 on Fig. 1: pops v1, v8, v10, v12, v9; then C's closest
+    is v4, worse than v10; returns v12, v9, v8, v10."""
+    ex = g1["ex1"]
+    r = oracle.alg1(g1["nbr"], g1["X"], g1["q"], k=4, entry=0)
+    assert r["pops"].tolist() == ex["pops"]
+    assert r["cmin"] == ex["cmin"][0]
+    assert r["ids"].tolist() == ex["result"]
+    assert r["dist_comps"] == ex["dist_comps"][0]
+
+
+def test_g1_is_nsw_with_dmin2(g1):
+    """G1 is an NSW graph with d_min = 2: v7's neighbours are v1, v5
+    (forward) and v8 (backward).  Checks the fixture, not the oracle."""
+    nbr = g1["nbr"]
+    assert sorted(nbr[6][nbr[6] >= 0].tolist()) == [0, 4, 7]
+    for v in range(12):
+        row = set(nbr[v][nbr[v] >= 0].tolist())
+        for u in row:
+            assert v in set(nbr[u][nbr[u] >= 0].tolist())   # bidirectional links
+        fwd = [u for u in row if u < v]
+        assert len(fwd) == min(2, v) or len(fwd) >= 2
+
+
+# ---------------------------------------------------- P4: brute force (O6)
+@pytest.mark.parametrize("metric", ["l2", "ip"])
+def test_bruteforce_matches_lexsort(metric):
+    for seed in range(20):
+        X = syn.random_int_points(60, 5, 0, 3, seed)        # heavy ties
+        Q = syn.random_int_points(7, 5, 0, 3, 100 + seed)
+        ids, dists = oracle.bruteforce(X, Q, k=9, metric=metric, threads=2)
+        for qi in range(len(Q)):
+            diff = X.astype(np.int64) - Q[qi].astype(np.int64)
+            dd = (diff ** 2).sum(1) if metric == "l2" else -(X.astype(np.int64) @ Q[qi].astype(np.int64))
+            order = np.lexsort((np.arange(len(X)), dd))[:9]
+            assert ids[qi].tolist() == order.tolist()
+            assert dists[qi].tolist() == dd[order].astype(np.float32).tolist()
+
+
+# ------------------------------------- P3: search == brute force when l >= n
+def _strongly_connected_graph(n, d_max, seed):
+    adj = syn.random_graph(n, d_max, seed, min_degree=1)
+    # a Hamiltonian cycle in slot 0 makes every vertex reachable from any entry
+    for v in range(n):
+        row = [u for u in adj[v].tolist() if u >= 0 and u != (v + 1) % n]
+        row = [(v + 1) % n] + row
+        adj[v] = (row + [-1] * d_max)[:d_max]
+    return adj
+
+
+@pytest.mark.parametrize("metric", ["l2", "ip"])
+def test_search_exact_when_l_ge_n(metric):
+    for seed in range(30):
+        n = 20 + seed % 17
+        X = syn.random_int_points(n, 4, 0, 4, seed)
+        Q = syn.random_int_points(3, 4, 0, 4, 500 + seed)
+        nbr = _strongly_connected_graph(n, 4, seed)
+        l = n + seed % 3
+        for k in (1, 5, n - 1):
+            ids, dists = oracle.search(nbr, X, Q, k=k, l=l, entry=seed % n, metric=metric)
+            gi, gd = oracle.bruteforce(X, Q, k=k, metric=metric, threads=1)
+            assert (ids == gi).all() and (dists == gd).all()
+
+
+# --------------------------------------------------- P5: search invariants
+def test_search_invariants_tie_heavy():
+    """Per-iteration invariants on 1500 tie-heavy random digraphs."""
+    rng = np.random.default_rng(5)
+    checked = 0
+    for seed in range(1500):
+        n = int(rng.integers(3, 30))
+        d_max = int(rng.integers(1, 6))
+        X = syn.random_int_points(n, 2, 0, 2, seed)          # distances in 0..8
+        q = syn.random_int_points(1, 2, 0, 2, 10_000 + seed)[0]
+        nbr = syn.random_graph(n, min(d_max, n - 1), seed, min_degree=0)
+        l = int(rng.integers(1, 17))
+        e = int(rng.integers(1, l + 1))
+        k = int(rng.integers(1, l + 1))
+        entry = int(rng.integers(0, n))
+        tr = oracle.search_trace(nbr, X, q, k=k, l=l, e=e, entry=entry)
+        dist = ((X.astype(np.int64) - q.astype(np.int64)) ** 2).sum(1)
+        explored = tr["explored"].tolist()
+        assert len(explored) == len(set(explored))              # never explored twice
+        assert len(explored) <= n
+        prev_worst = None
+        prev_N, prev_F = [entry], [0]
+        comps = 1
+        for i, v in enumerate(explored):
+            # v was the first unexplored entry among the first e of the previous N
+            cand = [u for u, f in zip(prev_N[:e], prev_F[:e]) if not f]
+            assert cand and cand[0] == v
+            N = [u for u in tr["N"][i].tolist() if u >= 0]
+            F = tr["flags"][i][:len(N)].tolist()
+            keys = [(dist[u], u) for u in N]
+            assert keys == sorted(keys) and len(set(N)) == len(N) and len(N) <= l
+            if len(N) == l:
+                if prev_worst is not None:
+                    assert keys[-1] <= prev_worst                 # l-th key never increases
+                prev_worst = keys[-1]
+            # explored flags survive; new entries are unexplored
+            for u, f in zip(N, F):
+                was = u == v or (u in prev_N and prev_F[prev_N.index(u)] == 1)
+                assert f == int(was)
+            # N is the l smallest of prev_N ∪ valid neighbours (a set)
+            row = [u for u in nbr[v].tolist() if u >= 0]
+            comps += len(row)
+            union = sorted(set(prev_N) | set(row), key=lambda u: (dist[u], u))[:l]
+            assert N == union
+            prev_N, prev_F = N, F
+        # termination: no unexplored entry among the first e
+        assert explored and all(prev_F[:e])
+        assert int(tr["stats"][0]) == len(explored)
+        assert int(tr["stats"][1]) == comps
+        out = [u for u in tr["ids"].tolist() if u >= 0]
+        assert out == prev_N[:k]
+        checked += 1
+    assert checked == 1500
+
+
+# -------------------------------------------- NSW definition
+def test_nsw_seq_exact_definition():
+    """Sequential NSW with exact NN: v's forward edges are its d_min nearest among
+    earlier points (all of them if fewer), links are bidirectional; checked with
+    an independent numpy lexsort."""
+    for seed in range(10):
+        n, d_min = 25, 3
+        X = syn.random_int_points(n, 3, 0, 3, seed)
+        ids, dists, _ = oracle.nsw_seq(X, d_min, n - 1, exact=True)
+        D = ((X[:, None, :].astype(np.int64) - X[None].astype(np.int64)) ** 2).sum(-1)
+        for v in range(n):
+            fwd = np.lexsort((np.arange(v), D[v, :v]))[:d_min].tolist() if v else []
+            row = ids[v][ids[v] >= 0].tolist()
+            assert set(fwd) <= set(row)
+            expect = set(fwd) | {w for w in range(v + 1, n)
+                                 if v in np.lexsort((np.arange(w), D[w, :w]))[:d_min]}
+            assert set(row) == expect
+            keys = [(D[v, u], u) for u in row]
+            assert keys == sorted(keys)
+            assert dists[v][:len(row)].tolist() == [float(D[v, u]) for u in row]
+
+
+# ----------------------------------- P6: quality theorem
+@pytest.mark.parametrize("metric", ["l2", "ip"])
+def test_alg2_equals_sequential_nsw_exact(metric):
+    rng = np.random.default_rng(3)
+    for seed in range(30):
+        n = int(rng.integers(20, 91))
+        d = int(rng.integers(2, 7))
+        d_min = int(rng.integers(2, 5))
+        d_max = 2 * d_min
+        X = syn.random_int_points(n, d, 0, 4, 300 + seed)
+        ref_i, ref_d, _ = oracle.nsw_seq(X, d_min, d_max, exact=True, metric=metric)
+        for s in (1, 3, 7, 16, n):
+            gi, gd, _ = oracle.alg2(X, d_min, d_max, s, exact=True, metric=metric)
+            assert (gi == ref_i).all(), (seed, s)
+            assert (gd == ref_d).all(), (seed, s)
+
+
+def test_alg2_equals_sequential_nsw_search_regime():
+    """Without an exact-NN hook: d_max >= n-1 (no truncation => connected) and
+    l_build >= n make every build search exact (P3), so the theorem applies to the
+    search-driven builds too.  This is the regime the GPU build is checked in."""
+    for seed in range(12):
+        n = 40 + seed
+        X = syn.random_int_points(n, 4, 0, 6, 700 + seed)
+        ref_i, _, _ = oracle.nsw_seq(X, 4, n - 1, exact=True)
+        seq_i, _, _ = oracle.nsw_seq(X, 4, n - 1, l_build=n + 1)
+        assert (seq_i == ref_i).all()
+        for s in (5, 16, n):
+            gi, _, _ = oracle.alg2(X, 4, n - 1, s, l_build=n + 1)
+            assert (gi == ref_i).all(), (seed, s)
+
+
+# ------------------------------------------------ P7: graph invariants
+def _check_graph_invariants(ids, dists, X, d_max, metric="l2"):
+    n = ids.shape[0]
+    for v in range(n):
+        row = ids[v].tolist()
+        c = sum(1 for u in row if u >= 0)
+        assert all(u >= 0 for u in row[:c]) and all(u == -1 for u in row[c:])  # -1 suffix
+        assert c <= d_max and v not in row[:c] and len(set(row[:c])) == c
+        keys = [(dists[v][j], row[j]) for j in range(c)]
+        assert keys == sorted(keys)
+        for j in range(0, c, max(1, c // 3)):
+            assert dists[v][j] == oracle.distance(X[v], X[row[j]], metric)
+
+
+def test_alg2_approx_invariants_and_groups():
+    X = syn.points(syn.with_size(syn.CONFIGS["C1"], n=1500))
+    for s in (64, 300, 1500):
+        ids, dists, st = oracle.alg2(X, 8, 16, s, l_build=32)
+        _check_graph_invariants(ids, dists, X, 16)
+        sizes = [min(s, 1500 - g) for g in range(0, 1500, s)]
+        assert st[2] == sum(z - 1 for z in sizes) + (1500 - sizes[0])   # searches run
+
+
+def test_alg2_max_rounds_zero_is_union_of_local_graphs():
+    X = syn.points(syn.with_size(syn.CONFIGS["C1"], n=900))
+    ids, _, _ = oracle.alg2(X, 8, 16, 300, l_build=32, max_rounds=0)
+    for g in range(3):
+        sub, _, _ = oracle.nsw_seq(X[g * 300:(g + 1) * 300], 8, 16, l_build=32)
+        sub = np.where(sub >= 0, sub + g * 300, -1)
+        assert (ids[g * 300:(g + 1) * 300] == sub).all()
+
+
+# ------------------------------------- P8: Fig. 12 quality (statistical)
+def test_alg2_quality_matches_sequential_nsw():
+    """Fig. 12: GGraphCon's graph is as good as the sequential NSW
+    graph; GNaiveParallel's is worse."""
+    cfg = syn.with_size(syn.CONFIGS["C1"], n=4000, nq=100)
+    X, Q = syn.points(cfg), syn.queries(cfg)
+    gt, _ = oracle.bruteforce(X, Q, 10)
+    seq, _, _ = oracle.nsw_seq(X, 8, 16, l_build=32)
+    a2, _, _ = oracle.alg2(X, 8, 16, 128, l_build=32)
+    nv, _ = oracle.naive_parallel(X, 8, 16, 500, l_build=32)
+    rec = {}
+    for name, g in (("seq", seq), ("alg2", a2), ("naive", nv)):
+        ids, _ = oracle.search(g, X, Q, k=10, l=32, threads=4)
+        rec[name] = oracle.recall(ids, gt)
+    assert abs(rec["alg2"] - rec["seq"]) <= 0.03, rec
+    assert rec["naive"] < rec["alg2"] - 0.02, rec
