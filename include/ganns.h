@@ -1,0 +1,168 @@
+/*
+ * ganns.h -- C ABI of the B200-native GANNS search / GGraphCon NSW construction
+ * library (libganns.so).  Yu, Wen, Zhang, Qin, Zhang, Lin, "GPU-accelerated
+ * Proximity Graph Approximate Nearest Neighbor Search and Construction",
+ * ICDE 2022.  "P:NNN" = line NNN of the paper text.
+ *
+ * Conventions for every entry point
+ *  - Plain C types only.  `stream` is a cudaStream_t passed as void* (NULL =
+ *    the legacy default stream).  Device pointers are CUDA global memory on the
+ *    graph's device; host pointers are ordinary (optionally pinned) memory.
+ *  - Vectors are fp32, row-major, rows of d floats, 16-byte aligned, d % 4 == 0.
+ *  - Ids are int32 vertex numbers = row index in `points` = insertion order
+ *    (P:260).  -1 marks an empty slot.
+ *  - Every function returns a ganns_status (0 = OK, < 0 = error) and never
+ *    throws or aborts; ganns_last_error() describes the last failure of the
+ *    calling thread.  On error no output is guaranteed to be written.
+ *  - Asynchronous on `stream` unless stated ("syncs").
+ *  - Results are deterministic: the same inputs give bit-identical outputs on
+ *    every run, stream and GPU count.
+ */
+#ifndef GANNS_H
+#define GANNS_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* Distance delta(q, x) (Table I: "Euclidean" and "Cosine Similarity").
+ *  GANNS_L2     squared Euclidean sum_j (q_j - x_j)^2 (same ranking as Euclidean)
+ *  GANNS_IP     -<q, x>
+ *  GANNS_COSINE 1 - <q, x> / ||q||; the caller passes unit-normalised `points`.
+ *               Inside ganns_build, COSINE orders candidates by -<x_v, x_u>
+ *               (identical ranking for unit rows, symmetric in u and v). */
+typedef enum { GANNS_L2 = 0, GANNS_IP = 1, GANNS_COSINE = 2 } ganns_metric;
+
+typedef enum {
+    GANNS_OK = 0,
+    GANNS_EINVAL = -1,   /* argument outside the documented domain */
+    GANNS_ENOMEM = -2,   /* device or host allocation failed */
+    GANNS_ECUDA = -3,    /* a CUDA runtime error (message has the CUDA string) */
+    GANNS_ENOTSUP = -4,  /* valid but unsupported combination */
+    GANNS_EIO = -5       /* file could not be read / written / has a bad header */
+} ganns_status;
+
+/* Opaque graph handle, library-owned.  Holds the fixed-degree adjacency
+ * int32 nbr[n][d_max] in device memory (Def. 2: directed, out-lists
+ * bounded by d_max; P:197 graph kept in GPU global memory) and its metadata.
+ * It does NOT hold or copy the point vectors: every search must pass the same
+ * `points` the graph was built from (a precondition that cannot be checked). */
+typedef struct ganns_graph ganns_graph;
+
+/* Parameters of Algorithm 2.  Zero-initialise for defaults. */
+typedef struct {
+    int d_min;          /* forward edges per vertex (Alg. 2 input P:316); 0 -> degree/2 */
+    int l_build;        /* candidate-array length of the build searches; 0 -> 64   */
+    int e_build;        /* explore budget of the build searches; 0 -> l_build      */
+    int64_t group_size; /* |P_i| of the partition (Alg. 2 line 1); 0 -> auto        */
+    int max_rounds;     /* Phase-2 rounds to run; < 0 (default -1 via 0 here means all)     */
+    int stop_after_phase1; /* != 0: return the union of local graphs (parity hook)         */
+    uint64_t *stats;    /* host, nullable, [4]: search iterations, distance computations,
+                           searches, rounds -- filled when ganns_build returns             */
+} ganns_build_params;
+
+/* Extra search parameters.  Zero-initialise for defaults. */
+typedef struct {
+    int e;              /* explore budget: only N[0..e) is eligible; 0 -> l        */
+    int64_t entry;      /* start vertex v_s; 0 (default) = vertex 0, R-C4           */
+    uint32_t *stats;    /* device, nullable, [nq][3]: iterations, distance computations,
+                           lazy-check drops per query                                       */
+} ganns_search_params;
+
+/* ganns_build -- GGraphCon NSW construction, Algorithm 2 (§IV-B
+ * P:253-297).  Phase 1 builds one local NSW per group by sequential insertion
+ * (P:266-281), Phase 2 merges groups 1..t into G_0 round by round,
+ * every search being the GANNS search of ganns_search with (l_build, e_build).
+ *   points  device, [n][d] fp32, read only, must stay alive for later searches
+ *   n       number of points, d_min < n < 2^31
+ *   d       dimension, d % 4 == 0, 4 <= d <= 4096
+ *   metric  ganns_metric
+ *   degree  d_max, 2 <= degree <= 128
+ *   p       nullable (all defaults)
+ *   out     receives a new graph on the current device.  Syncs `stream`.
+ * Scratch (build-form adjacency with distances, G', E, offsets) is allocated
+ * and freed inside the call. */
+int ganns_build(const float *points, int64_t n, int d, int metric, int degree,
+                const ganns_build_params *p, void *stream, ganns_graph **out);
+
+/* ganns_search -- batched GANNS search (§III-B): for each query,
+ * the k approximate nearest neighbours (Def. 1) found with a
+ * candidate array of length l (lazy update) and the lazy check.
+ *   g         graph
+ *   points    device [n][d], the vectors the graph was built from
+ *   queries   device [nq][d]
+ *   nq        >= 0 (0 is a no-op)
+ *   k         1 <= k <= l, k < n
+ *   l         k <= l <= 1024 (any value; not restricted to powers of two, R-C7)
+ *   out_ids   device [nq][k] int32, ascending (dist, id); -1 if fewer reachable (R-C8)
+ *   out_dists device [nq][k] fp32, +inf where out_ids is -1 */
+int ganns_search(const ganns_graph *g, const float *points, const float *queries, int64_t nq,
+                 int k, int l, int32_t *out_ids, float *out_dists, void *stream);
+
+/* ganns_search_ex -- ganns_search with explore budget e, entry vertex and
+ * per-query statistics (p nullable = ganns_search). */
+int ganns_search_ex(const ganns_graph *g, const float *points, const float *queries,
+                    int64_t nq, int k, int l, const ganns_search_params *p,
+                    int32_t *out_ids, float *out_dists, void *stream);
+
+/* ganns_search_host -- end-to-end search from HOST buffers (P:218 remark):
+ * queries_host [nq][d] is copied in, results are copied back to out_ids_host /
+ * out_dists_host [nq][k].  The batch is split in chunks pipelined over the
+ * library's copy/compute streams (H2D of chunk i+1 overlaps the search of
+ * chunk i and the D2H of chunk i-1).  Host buffers should be pinned
+ * (cudaHostAlloc / cudaHostRegister) for overlap.  Syncs. */
+int ganns_search_host(const ganns_graph *g, const float *points, const float *queries_host,
+                      int64_t nq, int k, int l, const ganns_search_params *p,
+                      int32_t *out_ids_host, float *out_dists_host, void *stream);
+
+/* ganns_merge_topk -- K6: merge W per-shard top-k lists into the global top-k
+ * (multi-GPU base-set sharding).  For each query the k smallest
+ * (dist, global id) over all shards.  All pointers device.
+ *   shard_ids   [W][nq][k] int32 GLOBAL ids (-1 = empty), shard_dists [W][nq][k]
+ *   out_ids / out_dists [nq][k]. */
+int ganns_merge_topk(const int32_t *shard_ids, const float *shard_dists, int W, int64_t nq,
+                     int k, int32_t *out_ids, float *out_dists, void *stream);
+
+/* ganns_offset_ids -- add `offset` to every id >= 0 of ids[count] (device),
+ * turning shard-local ids into global ids. */
+int ganns_offset_ids(int32_t *ids, int64_t count, int64_t offset, void *stream);
+
+/* ganns_graph_from_adjacency -- import an adjacency array (tests, oracle graphs).
+ *   nbr_host  host [n][d_max] int32; each row: distinct ids in [0, n), -1 padded
+ *             (rows with a repeated id are rejected: EINVAL)
+ *   d, metric metadata (the graph does not store vectors)
+ *   device    CUDA device ordinal for the copy.  Syncs. */
+int ganns_graph_from_adjacency(const int32_t *nbr_host, int64_t n, int d_max, int d,
+                               int metric, int device, ganns_graph **out);
+
+/* ganns_graph_adjacency -- copy the adjacency to host out_host [n][d_max].  Syncs. */
+int ganns_graph_adjacency(const ganns_graph *g, int32_t *out_host);
+
+/* ganns_graph_device_ptr -- device pointer to the adjacency [n][d_max] (borrowed). */
+int ganns_graph_device_ptr(const ganns_graph *g, const int32_t **nbr);
+
+/* ganns_graph_info -- any output pointer may be NULL. */
+int ganns_graph_info(const ganns_graph *g, int64_t *n, int *d, int *d_max, int *metric);
+
+/* ganns_graph_save / ganns_graph_load -- file = 32-byte header
+ * ("GANNSG01", n, d, d_max, metric) + int32 [n][d_max].  Syncs. */
+int ganns_graph_save(const ganns_graph *g, const char *path);
+int ganns_graph_load(const char *path, int device, ganns_graph **out);
+
+/* ganns_graph_free -- NULL is a no-op. */
+void ganns_graph_free(ganns_graph *g);
+
+/* ganns_last_error -- thread-local message of the last failing call ("" if none). */
+const char *ganns_last_error(void);
+
+/* ganns_kernel_launches -- number of kernels this library launched in this
+ * process so far (bench evidence for "gpu_launches"). */
+uint64_t ganns_kernel_launches(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* GANNS_H */

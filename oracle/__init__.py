@@ -85,12 +85,13 @@ def distance(q, x, metric="l2") -> float:
 
 
 def search(nbr, X, Q, k, l, e=0, entry=0, metric="l2", threads=1, stats=False):
-    """O2 over a batch of queries.  Returns ids [nq,k], dists [nq,k] (+ stats [nq,3])."""
+    """O2 over a batch of queries.  Returns ids [nq,k], dists [nq,k] (+ stats [nq,4]:
+    iterations, distance computations, lazy-check drops, merged entries)."""
     nbr, X, Q = _i32(nbr), _f32(X), _f32(np.atleast_2d(Q))
     nq = Q.shape[0]
     ids = np.empty((nq, k), np.int32)
     dists = np.empty((nq, k), np.float32)
-    st = np.empty((nq, 3), np.uint32) if stats else None
+    st = np.empty((nq, 4), np.uint32) if stats else None
     _check(lib().ora_search_batch(_p(nbr), nbr.shape[0], nbr.shape[1], _p(X), X.shape[1],
                                   METRICS[metric], _p(Q), nq, k, l, e, entry, _p(ids),
                                   _p(dists), _p(st), threads))
@@ -108,7 +109,7 @@ def search_trace(nbr, X, q, k, l, e=0, entry=0, metric="l2", max_iters=None):
     tr = np.full((max_iters, 1 + 2 * l + dm), -7, np.int32)
     ids = np.empty(k, np.int32)
     dists = np.empty(k, np.float32)
-    st = np.empty(3, np.uint32)
+    st = np.empty(4, np.uint32)
     _check(lib().ora_search_one(_p(nbr), nbr.shape[0], nbr.shape[1], _p(X), X.shape[1],
                                 METRICS[metric], _p(q), k, l, e, entry, _p(ids), _p(dists),
                                 _p(st), _p(tr), max_iters))
