@@ -24,6 +24,12 @@
 #include <stddef.h>
 #include <stdint.h>
 
+#if defined(__GNUC__)
+#define GANNS_API __attribute__((visibility("default")))
+#else
+#define GANNS_API
+#endif
+
 #ifdef __cplusplus
 extern "C" {
 #endif
@@ -58,7 +64,7 @@ typedef struct {
     int l_build;        /* candidate-array length of the build searches; 0 -> 64   */
     int e_build;        /* explore budget of the build searches; 0 -> l_build      */
     int64_t group_size; /* |P_i| of the partition (Alg. 2 line 1); 0 -> auto        */
-    int max_rounds;     /* Phase-2 rounds to run; < 0 (default -1 via 0 here means all)     */
+    int max_rounds;     /* 0 -> all t Phase-2 rounds; > 0 -> at most that many (parity hook) */
     int stop_after_phase1; /* != 0: return the union of local graphs (parity hook)         */
     uint64_t *stats;    /* host, nullable, [4]: search iterations, distance computations,
                            searches, rounds -- filled when ganns_build returns             */
@@ -68,8 +74,9 @@ typedef struct {
 typedef struct {
     int e;              /* explore budget: only N[0..e) is eligible; 0 -> l        */
     int64_t entry;      /* start vertex v_s; 0 (default) = vertex 0, R-C4           */
-    uint32_t *stats;    /* device, nullable, [nq][3]: iterations, distance computations,
-                           lazy-check drops per query                                       */
+    uint32_t *stats;    /* device, nullable, [nq][3] per query: iterations, distance
+                           computations (entry + every valid neighbour), T entries
+                           merged into N (kept among the first l)                   */
 } ganns_search_params;
 
 /* ganns_build -- GGraphCon NSW construction, Algorithm 2 (§IV-B
@@ -78,14 +85,14 @@ typedef struct {
  * every search being the GANNS search of ganns_search with (l_build, e_build).
  *   points  device, [n][d] fp32, read only, must stay alive for later searches
  *   n       number of points, d_min < n < 2^31
- *   d       dimension, d % 4 == 0, 4 <= d <= 4096
+ *   d       dimension, d % 4 == 0, 4 <= d <= 1024
  *   metric  ganns_metric
  *   degree  d_max, 2 <= degree <= 128
  *   p       nullable (all defaults)
  *   out     receives a new graph on the current device.  Syncs `stream`.
  * Scratch (build-form adjacency with distances, G', E, offsets) is allocated
  * and freed inside the call. */
-int ganns_build(const float *points, int64_t n, int d, int metric, int degree,
+GANNS_API int ganns_build(const float *points, int64_t n, int d, int metric, int degree,
                 const ganns_build_params *p, void *stream, ganns_graph **out);
 
 /* ganns_search -- batched GANNS search (§III-B): for each query,
@@ -99,12 +106,12 @@ int ganns_build(const float *points, int64_t n, int d, int metric, int degree,
  *   l         k <= l <= 1024 (any value; not restricted to powers of two, R-C7)
  *   out_ids   device [nq][k] int32, ascending (dist, id); -1 if fewer reachable (R-C8)
  *   out_dists device [nq][k] fp32, +inf where out_ids is -1 */
-int ganns_search(const ganns_graph *g, const float *points, const float *queries, int64_t nq,
+GANNS_API int ganns_search(const ganns_graph *g, const float *points, const float *queries, int64_t nq,
                  int k, int l, int32_t *out_ids, float *out_dists, void *stream);
 
 /* ganns_search_ex -- ganns_search with explore budget e, entry vertex and
  * per-query statistics (p nullable = ganns_search). */
-int ganns_search_ex(const ganns_graph *g, const float *points, const float *queries,
+GANNS_API int ganns_search_ex(const ganns_graph *g, const float *points, const float *queries,
                     int64_t nq, int k, int l, const ganns_search_params *p,
                     int32_t *out_ids, float *out_dists, void *stream);
 
@@ -114,7 +121,7 @@ int ganns_search_ex(const ganns_graph *g, const float *points, const float *quer
  * library's copy/compute streams (H2D of chunk i+1 overlaps the search of
  * chunk i and the D2H of chunk i-1).  Host buffers should be pinned
  * (cudaHostAlloc / cudaHostRegister) for overlap.  Syncs. */
-int ganns_search_host(const ganns_graph *g, const float *points, const float *queries_host,
+GANNS_API int ganns_search_host(const ganns_graph *g, const float *points, const float *queries_host,
                       int64_t nq, int k, int l, const ganns_search_params *p,
                       int32_t *out_ids_host, float *out_dists_host, void *stream);
 
@@ -123,44 +130,44 @@ int ganns_search_host(const ganns_graph *g, const float *points, const float *qu
  * (dist, global id) over all shards.  All pointers device.
  *   shard_ids   [W][nq][k] int32 GLOBAL ids (-1 = empty), shard_dists [W][nq][k]
  *   out_ids / out_dists [nq][k]. */
-int ganns_merge_topk(const int32_t *shard_ids, const float *shard_dists, int W, int64_t nq,
+GANNS_API int ganns_merge_topk(const int32_t *shard_ids, const float *shard_dists, int W, int64_t nq,
                      int k, int32_t *out_ids, float *out_dists, void *stream);
 
 /* ganns_offset_ids -- add `offset` to every id >= 0 of ids[count] (device),
  * turning shard-local ids into global ids. */
-int ganns_offset_ids(int32_t *ids, int64_t count, int64_t offset, void *stream);
+GANNS_API int ganns_offset_ids(int32_t *ids, int64_t count, int64_t offset, void *stream);
 
 /* ganns_graph_from_adjacency -- import an adjacency array (tests, oracle graphs).
  *   nbr_host  host [n][d_max] int32; each row: distinct ids in [0, n), -1 padded
  *             (rows with a repeated id are rejected: EINVAL)
  *   d, metric metadata (the graph does not store vectors)
  *   device    CUDA device ordinal for the copy.  Syncs. */
-int ganns_graph_from_adjacency(const int32_t *nbr_host, int64_t n, int d_max, int d,
+GANNS_API int ganns_graph_from_adjacency(const int32_t *nbr_host, int64_t n, int d_max, int d,
                                int metric, int device, ganns_graph **out);
 
 /* ganns_graph_adjacency -- copy the adjacency to host out_host [n][d_max].  Syncs. */
-int ganns_graph_adjacency(const ganns_graph *g, int32_t *out_host);
+GANNS_API int ganns_graph_adjacency(const ganns_graph *g, int32_t *out_host);
 
 /* ganns_graph_device_ptr -- device pointer to the adjacency [n][d_max] (borrowed). */
-int ganns_graph_device_ptr(const ganns_graph *g, const int32_t **nbr);
+GANNS_API int ganns_graph_device_ptr(const ganns_graph *g, const int32_t **nbr);
 
 /* ganns_graph_info -- any output pointer may be NULL. */
-int ganns_graph_info(const ganns_graph *g, int64_t *n, int *d, int *d_max, int *metric);
+GANNS_API int ganns_graph_info(const ganns_graph *g, int64_t *n, int *d, int *d_max, int *metric);
 
 /* ganns_graph_save / ganns_graph_load -- file = 32-byte header
  * ("GANNSG01", n, d, d_max, metric) + int32 [n][d_max].  Syncs. */
-int ganns_graph_save(const ganns_graph *g, const char *path);
-int ganns_graph_load(const char *path, int device, ganns_graph **out);
+GANNS_API int ganns_graph_save(const ganns_graph *g, const char *path);
+GANNS_API int ganns_graph_load(const char *path, int device, ganns_graph **out);
 
 /* ganns_graph_free -- NULL is a no-op. */
-void ganns_graph_free(ganns_graph *g);
+GANNS_API void ganns_graph_free(ganns_graph *g);
 
 /* ganns_last_error -- thread-local message of the last failing call ("" if none). */
-const char *ganns_last_error(void);
+GANNS_API const char *ganns_last_error(void);
 
 /* ganns_kernel_launches -- number of kernels this library launched in this
  * process so far (bench evidence for "gpu_launches"). */
-uint64_t ganns_kernel_launches(void);
+GANNS_API uint64_t ganns_kernel_launches(void);
 
 #ifdef __cplusplus
 }

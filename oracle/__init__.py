@@ -52,7 +52,8 @@ def lib():
         _lib.ora_nsw_seq.argtypes = [P, i64, i32, i32, i32, i32, i32, i32, i32, P, P, P]
         _lib.ora_alg2.argtypes = [P, i64, i32, i32, i32, i32, i32, i32, i64, i32, i32, P, P, P]
         _lib.ora_naive_parallel.argtypes = [P, i64, i32, i32, i32, i32, i32, i32, i64, P, P]
-        for f in ("ora_search_one", "ora_search_batch", "ora_alg1", "ora_bruteforce",
+        _lib.ora_merge_topk.argtypes = [P, P, i32, i64, i32, P, P]
+        for f in ("ora_merge_topk", "ora_search_one", "ora_search_batch", "ora_alg1", "ora_bruteforce",
                   "ora_nsw_seq", "ora_alg2", "ora_naive_parallel"):
             getattr(_lib, f).restype = ct.c_int
     return _lib
@@ -191,3 +192,13 @@ def naive_parallel(X, d_min, d_max, batch, l_build=64, e_build=0, metric="l2"):
     _check(lib().ora_naive_parallel(_p(X), n, X.shape[1], METRICS[metric], d_min, d_max,
                                     l_build, e_build, batch, _p(ids), _p(dists)))
     return ids, dists
+
+
+def merge_topk(ids, dists):
+    """k smallest (dist, id) of W per-shard lists [W, nq, k] -> [nq, k]."""
+    ids, dists = _i32(ids), _f32(dists)
+    W, nq, k = ids.shape
+    oi = np.empty((nq, k), np.int32)
+    od = np.empty((nq, k), np.float32)
+    _check(lib().ora_merge_topk(_p(ids), _p(dists), W, nq, k, _p(oi), _p(od)))
+    return oi, od

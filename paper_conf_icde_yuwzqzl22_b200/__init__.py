@@ -1,0 +1,245 @@
+"""B200-native GANNS search and GGraphCon NSW construction (Yu et al., ICDE 2022).
+
+Thin Python binding over the C ABI of ``libganns.so`` (include/ganns.h):
+argument marshalling only -- every step of the search and of the build runs in
+the library's sm_100a kernels.  PyTorch supplies device memory and streams.
+There is no CPU fallback: if the library is missing, importing this package
+raises.  Build it with ``__graft_entry__.build()`` (or ``python
+paper_conf_icde_yuwzqzl22_b200/_build.py``).
+"""
+from __future__ import annotations
+
+import ctypes as ct
+import os
+
+import numpy as np
+import torch
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libganns.so")
+
+METRICS = {"l2": 0, "ip": 1, "cosine": 2}
+_METRIC_NAMES = {v: k for k, v in METRICS.items()}
+
+
+class GannsError(RuntimeError):
+    pass
+
+
+class _BuildParams(ct.Structure):
+    _fields_ = [("d_min", ct.c_int), ("l_build", ct.c_int), ("e_build", ct.c_int),
+                ("group_size", ct.c_int64), ("max_rounds", ct.c_int),
+                ("stop_after_phase1", ct.c_int), ("stats", ct.POINTER(ct.c_uint64))]
+
+
+class _SearchParams(ct.Structure):
+    _fields_ = [("e", ct.c_int), ("entry", ct.c_int64), ("stats", ct.c_void_p)]
+
+
+def _load():
+    if not os.path.exists(LIB_PATH):
+        raise ImportError(f"{LIB_PATH} is missing; build it with __graft_entry__.build() "
+                          "(there is no CPU fallback)")
+    lib = ct.CDLL(LIB_PATH)
+    P, i32, i64 = ct.c_void_p, ct.c_int, ct.c_int64
+    sig = {
+        "ganns_build": [P, i64, i32, i32, i32, ct.POINTER(_BuildParams), P, ct.POINTER(P)],
+        "ganns_search": [P, P, P, i64, i32, i32, P, P, P],
+        "ganns_search_ex": [P, P, P, i64, i32, i32, ct.POINTER(_SearchParams), P, P, P],
+        "ganns_search_host": [P, P, P, i64, i32, i32, ct.POINTER(_SearchParams), P, P, P],
+        "ganns_merge_topk": [P, P, i32, i64, i32, P, P, P],
+        "ganns_offset_ids": [P, i64, i64, P],
+        "ganns_graph_from_adjacency": [P, i64, i32, i32, i32, i32, ct.POINTER(P)],
+        "ganns_graph_adjacency": [P, P],
+        "ganns_graph_device_ptr": [P, ct.POINTER(P)],
+        "ganns_graph_info": [P, ct.POINTER(i64), ct.POINTER(i32), ct.POINTER(i32), ct.POINTER(i32)],
+        "ganns_graph_save": [P, ct.c_char_p],
+        "ganns_graph_load": [ct.c_char_p, i32, ct.POINTER(P)],
+    }
+    for name, args in sig.items():
+        f = getattr(lib, name)
+        f.argtypes = args
+        f.restype = ct.c_int
+    lib.ganns_graph_free.argtypes = [P]
+    lib.ganns_graph_free.restype = None
+    lib.ganns_last_error.argtypes = []
+    lib.ganns_last_error.restype = ct.c_char_p
+    lib.ganns_kernel_launches.argtypes = []
+    lib.ganns_kernel_launches.restype = ct.c_uint64
+    return lib
+
+
+_lib = _load()
+
+# exported symbol list (include/ganns.h) -- checked by the CPU tests
+ABI_SYMBOLS = ("ganns_build", "ganns_search", "ganns_search_ex", "ganns_search_host",
+               "ganns_merge_topk", "ganns_offset_ids", "ganns_graph_from_adjacency",
+               "ganns_graph_adjacency", "ganns_graph_device_ptr", "ganns_graph_info",
+               "ganns_graph_save", "ganns_graph_load", "ganns_graph_free", "ganns_last_error",
+               "ganns_kernel_launches")
+
+
+def lib():
+    return _lib
+
+
+def _check(rc: int):
+    if rc != 0:
+        msg = _lib.ganns_last_error().decode(errors="replace")
+        raise GannsError(f"ganns error {rc}: {msg}")
+
+
+def _stream(stream) -> ct.c_void_p:
+    if stream is None:
+        stream = torch.cuda.current_stream()
+    return ct.c_void_p(stream.cuda_stream)
+
+
+def _dev_f32(t: torch.Tensor, name: str) -> torch.Tensor:
+    if not (isinstance(t, torch.Tensor) and t.is_cuda and t.dtype == torch.float32 and t.dim() == 2):
+        raise TypeError(f"{name} must be a 2-D float32 CUDA tensor")
+    return t.contiguous()
+
+
+def kernel_launches() -> int:
+    """Kernels launched by libganns.so in this process."""
+    return int(_lib.ganns_kernel_launches())
+
+
+class Graph:
+    """Fixed-degree proximity graph (int32 [n][d_max] adjacency in device memory)."""
+
+    def __init__(self, handle: ct.c_void_p):
+        self._h = handle
+        n, d, dm, m = ct.c_int64(), ct.c_int(), ct.c_int(), ct.c_int()
+        _check(_lib.ganns_graph_info(handle, ct.byref(n), ct.byref(d), ct.byref(dm), ct.byref(m)))
+        self.n, self.d, self.d_max, self.metric = n.value, d.value, dm.value, _METRIC_NAMES[m.value]
+        self.build_stats = None
+
+    @property
+    def handle(self):
+        return self._h
+
+    def adjacency(self) -> np.ndarray:
+        out = np.empty((self.n, self.d_max), np.int32)
+        _check(_lib.ganns_graph_adjacency(self._h, out.ctypes.data_as(ct.c_void_p)))
+        return out
+
+    def device_adjacency(self) -> int:
+        p = ct.c_void_p()
+        _check(_lib.ganns_graph_device_ptr(self._h, ct.byref(p)))
+        return p.value
+
+    def save(self, path: str):
+        _check(_lib.ganns_graph_save(self._h, path.encode()))
+
+    @staticmethod
+    def load(path: str, device: int = 0) -> "Graph":
+        h = ct.c_void_p()
+        _check(_lib.ganns_graph_load(path.encode(), device, ct.byref(h)))
+        return Graph(h)
+
+    def free(self):
+        if self._h:
+            _lib.ganns_graph_free(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.free()
+        except Exception:
+            pass
+
+
+def from_adjacency(nbr: np.ndarray, d: int, metric: str = "l2", device: int = 0) -> Graph:
+    nbr = np.ascontiguousarray(nbr, dtype=np.int32)
+    h = ct.c_void_p()
+    _check(_lib.ganns_graph_from_adjacency(nbr.ctypes.data_as(ct.c_void_p), nbr.shape[0],
+                                           nbr.shape[1], d, METRICS[metric], device, ct.byref(h)))
+    return Graph(h)
+
+
+def build(points: torch.Tensor, metric: str = "l2", degree: int = 32, d_min: int = 0,
+          l_build: int = 0, e_build: int = 0, group_size: int = 0, max_rounds: int = 0,
+          stop_after_phase1: bool = False, stream=None) -> Graph:
+    """GGraphCon NSW construction (Algorithm 2).  ``points`` [n, d] float32 CUDA
+    (unit rows for metric="cosine").  Returns a Graph; ``graph.build_stats`` =
+    (search iterations, distance computations, searches, rounds)."""
+    points = _dev_f32(points, "points")
+    st = (ct.c_uint64 * 4)()
+    p = _BuildParams(d_min, l_build, e_build, group_size, max_rounds, int(stop_after_phase1),
+                     ct.cast(st, ct.POINTER(ct.c_uint64)))
+    h = ct.c_void_p()
+    with torch.cuda.device(points.device):
+        _check(_lib.ganns_build(ct.c_void_p(points.data_ptr()), points.shape[0], points.shape[1],
+                                METRICS[metric], degree, ct.byref(p), _stream(stream), ct.byref(h)))
+    g = Graph(h)
+    g.build_stats = tuple(int(x) for x in st)
+    return g
+
+
+def search(graph: Graph, points: torch.Tensor, queries: torch.Tensor, k: int, l: int,
+           e: int = 0, entry: int = 0, stats: bool = False, out=None, stream=None):
+    """Batched GANNS search.  Returns (ids int32 [nq,k], dists float32 [nq,k]) on the
+    queries' device, plus per-query stats int32 [nq,3] (iterations, distance
+    computations, merged entries) when ``stats``."""
+    points = _dev_f32(points, "points")
+    queries = _dev_f32(queries, "queries")
+    nq = queries.shape[0]
+    if out is None:
+        ids = torch.empty((nq, k), dtype=torch.int32, device=queries.device)
+        dists = torch.empty((nq, k), dtype=torch.float32, device=queries.device)
+    else:
+        ids, dists = out
+    st = torch.empty((nq, 3), dtype=torch.int32, device=queries.device) if stats else None
+    p = _SearchParams(e, entry, ct.c_void_p(st.data_ptr()) if stats else None)
+    with torch.cuda.device(queries.device):
+        _check(_lib.ganns_search_ex(graph.handle, ct.c_void_p(points.data_ptr()),
+                                    ct.c_void_p(queries.data_ptr()), nq, k, l, ct.byref(p),
+                                    ct.c_void_p(ids.data_ptr()), ct.c_void_p(dists.data_ptr()),
+                                    _stream(stream)))
+    return (ids, dists, st) if stats else (ids, dists)
+
+
+def search_host(graph: Graph, points: torch.Tensor, queries: torch.Tensor, k: int, l: int,
+                e: int = 0, entry: int = 0, out=None, stream=None):
+    """End-to-end search from host memory: ``queries`` is a CPU float32 tensor
+    (pin it for copy/compute overlap); results come back in CPU tensors."""
+    points = _dev_f32(points, "points")
+    if queries.is_cuda or queries.dtype != torch.float32:
+        raise TypeError("queries must be a float32 CPU tensor")
+    queries = queries.contiguous()
+    nq = queries.shape[0]
+    if out is None:
+        ids = torch.empty((nq, k), dtype=torch.int32, pin_memory=True)
+        dists = torch.empty((nq, k), dtype=torch.float32, pin_memory=True)
+    else:
+        ids, dists = out
+    p = _SearchParams(e, entry, None)
+    with torch.cuda.device(points.device):
+        _check(_lib.ganns_search_host(graph.handle, ct.c_void_p(points.data_ptr()),
+                                      ct.c_void_p(queries.data_ptr()), nq, k, l, ct.byref(p),
+                                      ct.c_void_p(ids.data_ptr()), ct.c_void_p(dists.data_ptr()),
+                                      _stream(stream)))
+    return ids, dists
+
+
+def merge_topk(shard_ids: torch.Tensor, shard_dists: torch.Tensor, stream=None):
+    """K6: [W, nq, k] per-shard lists with GLOBAL ids -> global top-k [nq, k]."""
+    W, nq, k = shard_ids.shape
+    ids = torch.empty((nq, k), dtype=torch.int32, device=shard_ids.device)
+    dists = torch.empty((nq, k), dtype=torch.float32, device=shard_ids.device)
+    with torch.cuda.device(shard_ids.device):
+        _check(_lib.ganns_merge_topk(ct.c_void_p(shard_ids.contiguous().data_ptr()),
+                                     ct.c_void_p(shard_dists.contiguous().data_ptr()), W, nq, k,
+                                     ct.c_void_p(ids.data_ptr()), ct.c_void_p(dists.data_ptr()),
+                                     _stream(stream)))
+    return ids, dists
+
+
+def offset_ids(ids: torch.Tensor, offset: int, stream=None) -> torch.Tensor:
+    """In place: id -> id + offset for every id >= 0."""
+    with torch.cuda.device(ids.device):
+        _check(_lib.ganns_offset_ids(ct.c_void_p(ids.data_ptr()), ids.numel(), offset,
+                                     _stream(stream)))
+    return ids

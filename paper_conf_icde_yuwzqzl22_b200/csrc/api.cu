@@ -1,0 +1,377 @@
+// api.cu -- the C ABI of libganns.so (include/ganns.h): argument validation,
+// graph handles, error reporting, the host-buffer pipeline and save/load.
+// Every compute step runs in the kernels of search.cu / build.cu.
+#include "../../include/ganns.h"
+#include "ganns_internal.h"
+
+#include <algorithm>
+#include <cmath>
+#include <cstdio>
+#include <cstring>
+#include <mutex>
+#include <new>
+#include <vector>
+
+namespace ganns {
+
+static thread_local std::string g_last_error;
+static std::atomic<uint64_t> g_launches{0};
+
+void set_error(const std::string& msg) { g_last_error = msg; }
+int fail(int status, const std::string& msg) {
+  g_last_error = msg;
+  return status;
+}
+int cuda_fail(cudaError_t e, const char* what) {
+  return fail(GANNS_ECUDA, std::string(what) + ": " + cudaGetErrorString(e));
+}
+void count_launch(uint64_t n) { g_launches.fetch_add(n, std::memory_order_relaxed); }
+
+static bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
+
+static int check_graph(const ganns_graph* g) {
+  if (g == nullptr || g->nbr == nullptr) return fail(GANNS_EINVAL, "graph is NULL");
+  return GANNS_OK;
+}
+
+// Pipeline state for ganns_search_host: two streams and double-buffered device
+// staging, grown on demand (one set per device, guarded by a mutex).
+struct HostPipe {
+  int device = -1;
+  cudaStream_t st[2] = {nullptr, nullptr};
+  cudaEvent_t ev = nullptr;
+  float* dq[2] = {nullptr, nullptr};
+  int32_t* dids[2] = {nullptr, nullptr};
+  float* ddst[2] = {nullptr, nullptr};
+  size_t cap_q = 0, cap_r = 0;
+};
+static std::mutex g_pipe_mu;
+static HostPipe g_pipes[64];
+
+int run_build(BuildArgs& a, cudaStream_t s) {
+  switch (nv4_for(a.d)) {
+    case 1: return run_build_nv<1>(a, s);
+    case 2: return run_build_nv<2>(a, s);
+    case 4: return run_build_nv<4>(a, s);
+    case 8: return run_build_nv<8>(a, s);
+  }
+  return fail(GANNS_ENOTSUP, "unsupported dimension");
+}
+
+}  // namespace ganns
+
+using namespace ganns;
+
+extern "C" {
+
+const char* ganns_last_error(void) { return g_last_error.c_str(); }
+uint64_t ganns_kernel_launches(void) { return g_launches.load(); }
+
+int ganns_graph_info(const ganns_graph* g, int64_t* n, int* d, int* d_max, int* metric) {
+  if (int rc = check_graph(g)) return rc;
+  if (n) *n = g->n;
+  if (d) *d = g->d;
+  if (d_max) *d_max = g->d_max;
+  if (metric) *metric = g->metric;
+  return GANNS_OK;
+}
+
+int ganns_graph_device_ptr(const ganns_graph* g, const int32_t** nbr) {
+  if (int rc = check_graph(g)) return rc;
+  if (!nbr) return fail(GANNS_EINVAL, "nbr is NULL");
+  *nbr = g->nbr;
+  return GANNS_OK;
+}
+
+void ganns_graph_free(ganns_graph* g) {
+  if (!g) return;
+  if (g->nbr) {
+    int cur = 0;
+    cudaGetDevice(&cur);
+    cudaSetDevice(g->device);
+    cudaFree(g->nbr);
+    cudaSetDevice(cur);
+  }
+  delete g;
+}
+
+static int validate_common(int64_t n, int d, int metric, int d_max) {
+  if (n < 2 || n >= (int64_t(1) << 31)) return fail(GANNS_EINVAL, "n must be in [2, 2^31)");
+  if (d < 4 || d % 4 != 0 || d > 1024) return fail(GANNS_EINVAL, "d must be a multiple of 4 in [4, 1024]");
+  if (metric < 0 || metric > 2) return fail(GANNS_EINVAL, "unknown metric");
+  if (d_max < 2 || d_max > 128) return fail(GANNS_EINVAL, "degree must be in [2, 128]");
+  return GANNS_OK;
+}
+
+static int new_graph(int64_t n, int d, int d_max, int metric, ganns_graph** out) {
+  ganns_graph* g = new (std::nothrow) ganns_graph();
+  if (!g) return fail(GANNS_ENOMEM, "host allocation failed");
+  g->n = n;
+  g->d = d;
+  g->d_max = d_max;
+  g->metric = metric;
+  cudaGetDevice(&g->device);
+  cudaError_t e = cudaMalloc(&g->nbr, sizeof(int32_t) * size_t(n) * d_max);
+  if (e != cudaSuccess) {
+    delete g;
+    return fail(GANNS_ENOMEM, std::string("cudaMalloc(graph): ") + cudaGetErrorString(e));
+  }
+  *out = g;
+  return GANNS_OK;
+}
+
+int ganns_graph_from_adjacency(const int32_t* nbr_host, int64_t n, int d_max, int d, int metric,
+                               int device, ganns_graph** out) {
+  if (!nbr_host || !out) return fail(GANNS_EINVAL, "NULL argument");
+  if (int rc = validate_common(n, d, metric, d_max)) return rc;
+  std::vector<int32_t> seen(size_t(n), -1);   // row stamp per id
+  for (int64_t v = 0; v < n; ++v) {
+    for (int j = 0; j < d_max; ++j) {
+      int32_t u = nbr_host[size_t(v) * d_max + j];
+      if (u < -1 || u >= n) return fail(GANNS_EINVAL, "adjacency id out of range");
+      if (u < 0) continue;
+      if (seen[u] == int32_t(v)) return fail(GANNS_EINVAL, "adjacency row repeats an id");
+      seen[u] = int32_t(v);
+    }
+  }
+  int cur = 0;
+  cudaGetDevice(&cur);
+  if (cudaSetDevice(device) != cudaSuccess) return fail(GANNS_EINVAL, "bad device");
+  int rc = new_graph(n, d, d_max, metric, out);
+  if (rc == GANNS_OK) {
+    cudaError_t e = cudaMemcpy((*out)->nbr, nbr_host, sizeof(int32_t) * size_t(n) * d_max,
+                               cudaMemcpyHostToDevice);
+    if (e != cudaSuccess) {
+      ganns_graph_free(*out);
+      *out = nullptr;
+      rc = cuda_fail(e, "cudaMemcpy(adjacency)");
+    }
+  }
+  cudaSetDevice(cur);
+  return rc;
+}
+
+int ganns_graph_adjacency(const ganns_graph* g, int32_t* out_host) {
+  if (int rc = check_graph(g)) return rc;
+  if (!out_host) return fail(GANNS_EINVAL, "out is NULL");
+  cudaError_t e = cudaMemcpy(out_host, g->nbr, sizeof(int32_t) * size_t(g->n) * g->d_max,
+                             cudaMemcpyDeviceToHost);
+  return e == cudaSuccess ? GANNS_OK : cuda_fail(e, "cudaMemcpy(adjacency)");
+}
+
+int ganns_graph_save(const ganns_graph* g, const char* path) {
+  if (int rc = check_graph(g)) return rc;
+  if (!path) return fail(GANNS_EINVAL, "path is NULL");
+  std::vector<int32_t> h(size_t(g->n) * g->d_max);
+  if (int rc = ganns_graph_adjacency(g, h.data())) return rc;
+  FILE* f = std::fopen(path, "wb");
+  if (!f) return fail(GANNS_EIO, std::string("cannot open ") + path);
+  char magic[8] = {'G', 'A', 'N', 'N', 'S', 'G', '0', '1'};
+  int64_t n = g->n;
+  int32_t meta[4] = {g->d, g->d_max, g->metric, 0};
+  bool ok = std::fwrite(magic, 1, 8, f) == 8 && std::fwrite(&n, 8, 1, f) == 1 &&
+            std::fwrite(meta, 4, 4, f) == 4 && std::fwrite(h.data(), 4, h.size(), f) == h.size();
+  ok = (std::fclose(f) == 0) && ok;
+  return ok ? GANNS_OK : fail(GANNS_EIO, std::string("write failed: ") + path);
+}
+
+int ganns_graph_load(const char* path, int device, ganns_graph** out) {
+  if (!path || !out) return fail(GANNS_EINVAL, "NULL argument");
+  FILE* f = std::fopen(path, "rb");
+  if (!f) return fail(GANNS_EIO, std::string("cannot open ") + path);
+  char magic[8];
+  int64_t n = 0;
+  int32_t meta[4];
+  bool ok = std::fread(magic, 1, 8, f) == 8 && std::memcmp(magic, "GANNSG01", 8) == 0 &&
+            std::fread(&n, 8, 1, f) == 1 && std::fread(meta, 4, 4, f) == 4;
+  if (!ok || n < 2 || meta[1] < 2 || meta[1] > 128) {
+    std::fclose(f);
+    return fail(GANNS_EIO, std::string("bad graph header: ") + path);
+  }
+  std::vector<int32_t> h(size_t(n) * meta[1]);
+  ok = std::fread(h.data(), 4, h.size(), f) == h.size();
+  std::fclose(f);
+  if (!ok) return fail(GANNS_EIO, std::string("truncated graph file: ") + path);
+  return ganns_graph_from_adjacency(h.data(), n, meta[1], meta[0], meta[2], device, out);
+}
+
+static int validate_search(const ganns_graph* g, const float* points, const float* queries,
+                           int64_t nq, int k, int l, const ganns_search_params* p,
+                           const void* out_ids, const void* out_dists, int* e_out,
+                           int32_t* entry_out) {
+  if (int rc = check_graph(g)) return rc;
+  if (nq < 0) return fail(GANNS_EINVAL, "nq < 0");
+  if (k < 1 || k >= g->n) return fail(GANNS_EINVAL, "k must be in [1, n)");
+  if (l < k || l > 1024) return fail(GANNS_EINVAL, "l must be in [k, 1024]");
+  int e = p ? p->e : 0;
+  if (e < 0 || e > l) return fail(GANNS_EINVAL, "e must be in [0, l]");
+  int64_t entry = p ? p->entry : 0;
+  if (entry < 0 || entry >= g->n) return fail(GANNS_EINVAL, "entry out of range");
+  if (nq > 0 && (!points || !queries || !out_ids || !out_dists))
+    return fail(GANNS_EINVAL, "NULL pointer");
+  if (!aligned16(points) || !aligned16(queries)) return fail(GANNS_EINVAL, "points/queries not 16-byte aligned");
+  *e_out = e == 0 ? l : e;
+  *entry_out = int32_t(entry);
+  return GANNS_OK;
+}
+
+int ganns_search_ex(const ganns_graph* g, const float* points, const float* queries, int64_t nq,
+                    int k, int l, const ganns_search_params* p, int32_t* out_ids,
+                    float* out_dists, void* stream) {
+  int e = 0;
+  int32_t entry = 0;
+  if (int rc = validate_search(g, points, queries, nq, k, l, p, out_ids, out_dists, &e, &entry))
+    return rc;
+  if (nq == 0) return GANNS_OK;
+  SearchLaunch a{g->nbr, points, g->n, g->d, g->d_max, g->metric, queries, nq, k, l, e, entry,
+                 out_ids, out_dists, p ? p->stats : nullptr};
+  cudaError_t err = launch_search(a, static_cast<cudaStream_t>(stream));
+  return err == cudaSuccess ? GANNS_OK : cuda_fail(err, "search kernel launch");
+}
+
+int ganns_search(const ganns_graph* g, const float* points, const float* queries, int64_t nq,
+                 int k, int l, int32_t* out_ids, float* out_dists, void* stream) {
+  return ganns_search_ex(g, points, queries, nq, k, l, nullptr, out_ids, out_dists, stream);
+}
+
+int ganns_search_host(const ganns_graph* g, const float* points, const float* queries_host,
+                      int64_t nq, int k, int l, const ganns_search_params* p,
+                      int32_t* out_ids_host, float* out_dists_host, void* stream) {
+  int e = 0;
+  int32_t entry = 0;
+  if (int rc = validate_search(g, points, queries_host, nq, k, l, p, out_ids_host,
+                               out_dists_host, &e, &entry))
+    return rc;
+  if (p && p->stats) return fail(GANNS_EINVAL, "stats are not supported by ganns_search_host");
+  if (nq == 0) return GANNS_OK;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (dev < 0 || dev >= 64) return fail(GANNS_ENOTSUP, "device ordinal >= 64");
+  std::lock_guard<std::mutex> lock(g_pipe_mu);
+  HostPipe& P = g_pipes[dev];
+  if (P.device != dev) {
+    for (int i = 0; i < 2; ++i)
+      if (cudaStreamCreateWithFlags(&P.st[i], cudaStreamNonBlocking) != cudaSuccess)
+        return fail(GANNS_ECUDA, "cudaStreamCreate failed");
+    if (cudaEventCreateWithFlags(&P.ev, cudaEventDisableTiming) != cudaSuccess)
+      return fail(GANNS_ECUDA, "cudaEventCreate failed");
+    P.device = dev;
+  }
+  // chunking: at least 2 chunks to overlap copies with the search, each large
+  // enough to fill the GPU (~8 queries per SM warp slot).
+  int64_t chunk = std::max<int64_t>(2048, (nq + 3) / 4);
+  if (chunk > nq) chunk = nq;
+  const size_t need_q = size_t(chunk) * g->d, need_r = size_t(chunk) * k;
+  if (need_q > P.cap_q || need_r > P.cap_r) {
+    for (int i = 0; i < 2; ++i) {
+      cudaFree(P.dq[i]);
+      cudaFree(P.dids[i]);
+      cudaFree(P.ddst[i]);
+      P.dq[i] = nullptr;
+      P.dids[i] = nullptr;
+      P.ddst[i] = nullptr;
+    }
+    P.cap_q = P.cap_r = 0;
+    for (int i = 0; i < 2; ++i) {
+      if (cudaMalloc(&P.dq[i], need_q * sizeof(float)) != cudaSuccess ||
+          cudaMalloc(&P.dids[i], need_r * sizeof(int32_t)) != cudaSuccess ||
+          cudaMalloc(&P.ddst[i], need_r * sizeof(float)) != cudaSuccess)
+        return fail(GANNS_ENOMEM, "cudaMalloc(search_host staging)");
+    }
+    P.cap_q = need_q;
+    P.cap_r = need_r;
+  }
+  cudaStream_t user = static_cast<cudaStream_t>(stream);
+  cudaError_t err = cudaEventRecord(P.ev, user);
+  for (int i = 0; i < 2 && err == cudaSuccess; ++i) err = cudaStreamWaitEvent(P.st[i], P.ev, 0);
+  for (int64_t q0 = 0, c = 0; q0 < nq && err == cudaSuccess; q0 += chunk, ++c) {
+    const int64_t m = std::min(chunk, nq - q0);
+    const int b = int(c & 1);
+    cudaStream_t s = P.st[b];
+    err = cudaMemcpyAsync(P.dq[b], queries_host + size_t(q0) * g->d, sizeof(float) * m * g->d,
+                          cudaMemcpyHostToDevice, s);
+    if (err != cudaSuccess) break;
+    SearchLaunch a{g->nbr, points, g->n, g->d, g->d_max, g->metric, P.dq[b], m, k, l, e, entry,
+                   P.dids[b], P.ddst[b], nullptr};
+    err = launch_search(a, s);
+    if (err != cudaSuccess) break;
+    err = cudaMemcpyAsync(out_ids_host + size_t(q0) * k, P.dids[b], sizeof(int32_t) * m * k,
+                          cudaMemcpyDeviceToHost, s);
+    if (err == cudaSuccess)
+      err = cudaMemcpyAsync(out_dists_host + size_t(q0) * k, P.ddst[b], sizeof(float) * m * k,
+                            cudaMemcpyDeviceToHost, s);
+  }
+  for (int i = 0; i < 2; ++i) {
+    cudaError_t e2 = cudaStreamSynchronize(P.st[i]);
+    if (err == cudaSuccess) err = e2;
+  }
+  return err == cudaSuccess ? GANNS_OK : cuda_fail(err, "ganns_search_host");
+}
+
+
+int ganns_build(const float* points, int64_t n, int d, int metric, int degree,
+                const ganns_build_params* p, void* stream, ganns_graph** out) {
+  if (!points || !out) return fail(GANNS_EINVAL, "NULL argument");
+  if (int rc = validate_common(n, d, metric, degree)) return rc;
+  if (!aligned16(points)) return fail(GANNS_EINVAL, "points not 16-byte aligned");
+  int d_min = p && p->d_min > 0 ? p->d_min : degree / 2;
+  if (d_min < 1) d_min = 1;
+  int l_build = p && p->l_build > 0 ? p->l_build : 64;
+  int e_build = p && p->e_build > 0 ? p->e_build : l_build;
+  if (d_min > degree) return fail(GANNS_EINVAL, "d_min > degree");
+  if (d_min >= n) return fail(GANNS_EINVAL, "d_min must be < n");
+  if (l_build < d_min || l_build > 1024) return fail(GANNS_EINVAL, "l_build must be in [d_min, 1024]");
+  if (e_build < 1 || e_build > l_build) return fail(GANNS_EINVAL, "e_build must be in [1, l_build]");
+  int64_t S = p && p->group_size > 0 ? p->group_size : 0;
+  if (S == 0) {
+    // R-C14: clamp(pow2(2 sqrt n), 256, 8192)
+    double t = 2.0 * std::sqrt(double(n));
+    int64_t s2 = int64_t(1) << int64_t(std::llround(std::log2(std::max(t, 1.0))));
+    S = std::min<int64_t>(8192, std::max<int64_t>(256, s2));
+  }
+  if (S > n) S = n;
+  if (p && p->group_size < 0) return fail(GANNS_EINVAL, "group_size < 0");
+  int rc = new_graph(n, d, degree, metric, out);
+  if (rc) return rc;
+  BuildArgs a{};
+  a.X = points;
+  a.n = n;
+  a.d = d;
+  a.metric = metric == GANNS_COSINE ? GANNS_IP : metric;   // symmetric keys inside the build
+  a.d_max = degree;
+  a.d_min = d_min;
+  a.l_build = l_build;
+  a.e_build = e_build;
+  a.group_size = S;
+  a.max_rounds = p ? (p->stop_after_phase1 ? 0 : (p->max_rounds > 0 ? p->max_rounds : -1)) : -1;
+  a.out_nbr = (*out)->nbr;
+  rc = run_build(a, static_cast<cudaStream_t>(stream));
+  if (rc) {
+    ganns_graph_free(*out);
+    *out = nullptr;
+    return rc;
+  }
+  if (p && p->stats)
+    for (int i = 0; i < 4; ++i) p->stats[i] = a.stats[i];
+  return GANNS_OK;
+}
+
+int ganns_merge_topk(const int32_t* shard_ids, const float* shard_dists, int W, int64_t nq, int k,
+                     int32_t* out_ids, float* out_dists, void* stream) {
+  if (W < 1 || k < 1 || nq < 0) return fail(GANNS_EINVAL, "bad W / k / nq");
+  if (size_t(W) * k * kWarpsPerBlock * 8 > 200 * 1024) return fail(GANNS_ENOTSUP, "W*k too large");
+  if (nq > 0 && (!shard_ids || !shard_dists || !out_ids || !out_dists))
+    return fail(GANNS_EINVAL, "NULL pointer");
+  cudaError_t e = launch_merge_topk(shard_ids, shard_dists, W, nq, k, out_ids, out_dists,
+                                    static_cast<cudaStream_t>(stream));
+  return e == cudaSuccess ? GANNS_OK : cuda_fail(e, "merge_topk launch");
+}
+
+int ganns_offset_ids(int32_t* ids, int64_t count, int64_t offset, void* stream) {
+  if (count < 0 || (count > 0 && !ids)) return fail(GANNS_EINVAL, "bad ids/count");
+  if (offset < 0 || offset >= (int64_t(1) << 31)) return fail(GANNS_EINVAL, "offset out of range");
+  cudaError_t e = launch_offset_ids(ids, count, offset, static_cast<cudaStream_t>(stream));
+  return e == cudaSuccess ? GANNS_OK : cuda_fail(e, "offset_ids launch");
+}
+
+}  // extern "C"

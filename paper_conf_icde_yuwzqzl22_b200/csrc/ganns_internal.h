@@ -1,0 +1,68 @@
+// ganns_internal.h -- host-side declarations shared by the .cu translation units
+// of libganns.so (not part of the public ABI; see include/ganns.h).
+#pragma once
+#include <cuda_runtime.h>
+#include <atomic>
+#include <cstdint>
+#include <string>
+
+struct ganns_graph {
+  int32_t* nbr = nullptr;   // device [n][d_max]
+  int64_t n = 0;
+  int d = 0;
+  int d_max = 0;
+  int metric = 0;
+  int device = 0;
+};
+
+namespace ganns {
+
+constexpr int kWarpsPerBlock = 4;   // queries (warps) per CTA of the search kernel
+
+void set_error(const std::string& msg);
+int fail(int status, const std::string& msg);
+int cuda_fail(cudaError_t e, const char* what);
+void count_launch(uint64_t n = 1);
+
+// Template selectors.
+inline int nv4_for(int d) {
+  int d4 = d / 4;
+  return d4 <= 32 ? 1 : d4 <= 64 ? 2 : d4 <= 128 ? 4 : d4 <= 256 ? 8 : -1;
+}
+inline int tpl_for(int d_max) { return d_max <= 32 ? 1 : d_max <= 64 ? 2 : d_max <= 128 ? 4 : -1; }
+
+struct SearchLaunch {
+  const int32_t* nbr;
+  const float* X;
+  int64_t n;
+  int d, d_max, metric;
+  const float* Q;
+  int64_t nq;
+  int k, l, e;
+  int32_t entry;
+  int32_t* out_ids;
+  float* out_dists;
+  uint32_t* stats;
+};
+cudaError_t launch_search(const SearchLaunch& a, cudaStream_t s);
+template <int NV4>
+cudaError_t launch_search_nv(const SearchLaunch& a, cudaStream_t s);
+
+struct BuildArgs {
+  const float* X;
+  int64_t n;
+  int d, metric, d_max, d_min, l_build, e_build;
+  int64_t group_size;
+  int max_rounds;       // < 0: all
+  int32_t* out_nbr;     // device [n][d_max]
+  uint64_t stats[4];    // out: iterations, distance computations, searches, rounds
+};
+int run_build(BuildArgs& a, cudaStream_t s);
+template <int NV4>
+int run_build_nv(BuildArgs& a, cudaStream_t s);
+
+cudaError_t launch_merge_topk(const int32_t* ids, const float* dists, int W, int64_t nq, int k,
+                              int32_t* out_ids, float* out_dists, cudaStream_t s);
+cudaError_t launch_offset_ids(int32_t* ids, int64_t count, int64_t offset, cudaStream_t s);
+
+}  // namespace ganns

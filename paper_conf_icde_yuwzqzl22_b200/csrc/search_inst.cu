@@ -1,0 +1,78 @@
+// search_inst.cu -- K1 instantiations for one NV4 (= float4 per lane per row);
+// compiled once per NV4 in {1, 2, 4, 8} with -DGANNS_NV4=... so the template
+// instances build in parallel.  See ganns_dev.cuh for the algorithm.
+#include "ganns_dev.cuh"
+#include "ganns_internal.h"
+
+#ifndef GANNS_NV4
+#error "compile with -DGANNS_NV4=<1|2|4|8>"
+#endif
+
+namespace ganns {
+
+template <int NV4, int TPL, bool L2>
+__global__ void __launch_bounds__(kWarpsPerBlock * 32)
+search_kernel(GraphView g, const float* __restrict__ Q, int64_t nq, int k, int l, int e,
+              int32_t entry, int32_t* __restrict__ out_ids, float* __restrict__ out_dists,
+              uint32_t* __restrict__ stats) {
+  extern __shared__ __align__(16) uint8_t smem[];
+  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int64_t q = int64_t(blockIdx.x) * kWarpsPerBlock + w;
+  if (q >= nq) return;
+  uint8_t* base = smem + size_t(w) * warp_smem_bytes(l, TPL);
+  uint64_t* sN = reinterpret_cast<uint64_t*>(base);
+  uint64_t* sT = sN + lpad32(l);
+  uint32_t* sBM = reinterpret_cast<uint32_t*>(sT + TPL * 32);
+  SearchStats st;
+  const int cnt = warp_search<NV4, TPL, L2, false>(g, Q + size_t(q) * (g.d4 * 4), entry, l, e,
+                                                   sN, sT, sBM, st);
+  // output: the first k of N, (-1, +inf) padded (R-C8)
+  for (int i = lane; i < k; i += 32) {
+    uint64_t key = i < cnt ? unflag(sN[i]) : kKeyInf;
+    bool empty = key_empty(key);
+    out_ids[size_t(q) * k + i] = empty ? -1 : key_id(key);
+    out_dists[size_t(q) * k + i] = empty ? __int_as_float(0x7f800000) : key_dist(key);
+  }
+  if (stats != nullptr && lane == 0) {
+    stats[size_t(q) * 3 + 0] = st.iters;
+    stats[size_t(q) * 3 + 1] = st.comps;
+    stats[size_t(q) * 3 + 2] = st.merged;
+  }
+}
+
+template <int NV4, int TPL, bool L2>
+static cudaError_t launch_t(const SearchLaunch& a, cudaStream_t s) {
+  auto kern = search_kernel<NV4, TPL, L2>;
+  const size_t smem = size_t(kWarpsPerBlock) * warp_smem_bytes(a.l, TPL);
+  static bool attr_done = false;   // per instantiation
+  if (!attr_done) {
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         int(kWarpsPerBlock * warp_smem_bytes(1024, TPL)));
+    if (e != cudaSuccess) return e;
+    attr_done = true;
+  }
+  GraphView g{a.nbr, a.X, a.n, a.d_max, a.d / 4, a.metric};
+  const int64_t blocks = (a.nq + kWarpsPerBlock - 1) / kWarpsPerBlock;
+  kern<<<dim3(unsigned(blocks)), kWarpsPerBlock * 32, smem, s>>>(
+      g, a.Q, a.nq, a.k, a.l, a.e, a.entry, a.out_ids, a.out_dists, a.stats);
+  count_launch();
+  return cudaGetLastError();
+}
+
+template <int NV4, int TPL>
+static cudaError_t launch_m(const SearchLaunch& a, cudaStream_t s) {
+  return a.metric == 0 ? launch_t<NV4, TPL, true>(a, s) : launch_t<NV4, TPL, false>(a, s);
+}
+template <int NV4>
+cudaError_t launch_search_nv(const SearchLaunch& a, cudaStream_t s) {
+  switch (tpl_for(a.d_max)) {
+    case 1: return launch_m<NV4, 1>(a, s);
+    case 2: return launch_m<NV4, 2>(a, s);
+    case 4: return launch_m<NV4, 4>(a, s);
+  }
+  return cudaErrorInvalidValue;
+}
+
+template cudaError_t launch_search_nv<GANNS_NV4>(const SearchLaunch&, cudaStream_t);
+
+}  // namespace ganns

@@ -1,0 +1,51 @@
+"""Host-side checks that need no GPU: the C-ABI library loads and exports every
+symbol include/ganns.h declares; the product package does not reach the oracle."""
+import ctypes
+import os
+import re
+
+from conftest import ROOT
+
+HEADER = os.path.join(ROOT, "include", "ganns.h")
+LIB = os.path.join(ROOT, "paper_conf_icde_yuwzqzl22_b200", "libganns.so")
+
+
+def declared_symbols():
+    src = open(HEADER).read()
+    return sorted(set(re.findall(r"GANNS_API\s+[\w\s\*]*?\b(ganns_\w+)\s*\(", src)))
+
+
+def test_header_declares_the_north_star_calls():
+    syms = declared_symbols()
+    for s in ("ganns_build", "ganns_search"):
+        assert s in syms
+    assert len(syms) >= 15
+
+
+def test_library_loads_and_exports_every_declared_symbol():
+    lib = ctypes.CDLL(LIB)
+    for s in declared_symbols():
+        assert hasattr(lib, s), s
+
+
+def test_binding_lists_every_symbol():
+    import paper_conf_icde_yuwzqzl22_b200 as g
+    assert sorted(g.ABI_SYMBOLS) == declared_symbols()
+
+
+def test_product_path_never_imports_the_oracle():
+    pkg = os.path.join(ROOT, "paper_conf_icde_yuwzqzl22_b200")
+    for dirpath, _, files in os.walk(pkg):
+        for f in files:
+            if f.endswith((".py", ".cu", ".cuh", ".h", ".cpp")):
+                text = open(os.path.join(dirpath, f)).read()
+                assert "import oracle" not in text and "ganns_oracle" not in text, f
+                assert "from oracle" not in text, f
+
+
+def test_last_error_without_gpu_calls():
+    lib = ctypes.CDLL(LIB)
+    lib.ganns_last_error.restype = ctypes.c_char_p
+    lib.ganns_graph_info.restype = ctypes.c_int
+    assert lib.ganns_graph_info(None, None, None, None, None) == -1   # EINVAL on NULL graph
+    assert b"NULL" in lib.ganns_last_error()

@@ -292,3 +292,22 @@ def test_alg2_quality_matches_sequential_nsw():
         rec[name] = oracle.recall(ids, gt)
     assert abs(rec["alg2"] - rec["seq"]) <= 0.03, rec
     assert rec["naive"] < rec["alg2"] - 0.02, rec
+
+
+# ------------------------------- shard merge == global brute force
+@pytest.mark.parametrize("W", [1, 2, 3, 8])
+def test_merge_topk_of_exact_shards_is_global_bruteforce(W):
+    """If every shard returns its exact top-k, the merged top-k is the exact
+    top-k of the whole base set (Def. 1 on the union)."""
+    X = syn.random_int_points(400, 4, 0, 3, 41 + W)     # tie-heavy
+    Q = syn.random_int_points(9, 4, 0, 3, 99)
+    k = 12
+    bounds = np.linspace(0, len(X), W + 1).astype(int)
+    sid, sd = [], []
+    for a, b in zip(bounds[:-1], bounds[1:]):
+        i, d = oracle.bruteforce(X[a:b], Q, k, threads=1)
+        sid.append(np.where(i >= 0, i + a, -1))
+        sd.append(d)
+    mi, md = oracle.merge_topk(np.stack(sid), np.stack(sd))
+    gi, gd = oracle.bruteforce(X, Q, k, threads=1)
+    assert (mi == gi).all() and (md == gd).all()
