@@ -1,0 +1,394 @@
+#!/usr/bin/env python
+"""bench.py -- queries/sec at recall@10 = 0.95 on SIFT1M-shaped data (BASELINE.json
+configs[1]), plus GGraphCon NSW build seconds, on N B200s.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config C2] [--impl ours|reference]
+
+One step = one ganns_search launch over the whole 10K-query batch at the smallest
+l (from the sweep) whose recall@10 >= 0.95 -- the whole hot path (candidate
+locating, adjacency gather, bulk distance, lazy check, sort, merge, top-k out)
+in one fused kernel.  Inputs are resident in HBM when the timed region starts;
+L2 is flushed (256 MiB write) between timed steps.  Under torchrun each rank
+builds the same deterministic graph and searches its own batch of nq queries
+(weak scaling, no data-path collective); time = max over ranks.
+
+--impl reference times the CPU oracle (oracle/, plain C, all host cores) on a
+bounded sample of the same queries, same graph, same l.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import ganns_synth as syn  # noqa: E402
+
+L_SWEEP = [32, 40, 48, 56, 64, 80, 96, 112, 128, 160, 192, 256, 320, 384, 512]
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default="C2")
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--target", type=float, default=0.95)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=12.0)
+    ap.add_argument("--json-out", default=None)
+    return ap.parse_args()
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            m = json.load(f)
+        return float(m["hbm_gbs"]), "measured"
+    return 6650.0, "fallback"
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+
+    Q = ("index,clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.proc = None
+        self.lines = []
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.Q}",
+                 "--format=csv,noheader,nounits", "-lms", "100"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except FileNotFoundError:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except subprocess.TimeoutExpired:
+                self.proc.kill()
+
+    def summary(self):
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 7:
+                continue
+            try:
+                sm.append(float(f[1]))
+                mx = float(f[2])
+            except ValueError:
+                continue
+            for nm, v in zip(names, f[3:7]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": mx,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def make_workload(cfg, rank: int):
+    X = syn.points(cfg)
+    # every rank draws its own batch of nq queries (weak scaling); rank 0 = the config's
+    Qall = syn.queries(cfg, cfg.nq * (rank + 1))
+    Q = Qall[rank * cfg.nq:(rank + 1) * cfg.nq]
+    return X, np.ascontiguousarray(Q)
+
+
+def ground_truth(torch, Xd, Qd, k):
+    """Exact top-k by (dist, id) with torch fp32 matmuls on the GPU (bench-side
+    measurement only).  Integer-grid data: every term < 2^24, so exact."""
+    torch.backends.cuda.matmul.allow_tf32 = False
+    n = Xd.shape[0]
+    xn = (Xd.double() ** 2).sum(1).float()
+    qn = (Qd.double() ** 2).sum(1).float()
+    best = None
+    shift = 1 << 21
+    for a in range(0, n, 131072):
+        b = min(n, a + 131072)
+        D = qn[:, None] + xn[None, a:b] - 2.0 * (Qd @ Xd[a:b].T)
+        key = D.round().long() * shift + torch.arange(a, b, device=Xd.device)[None, :]
+        kk = torch.topk(key, k, dim=1, largest=False, sorted=True).values
+        best = kk if best is None else torch.topk(torch.cat([best, kk], 1), k, dim=1,
+                                                  largest=False, sorted=True).values
+    return (best % shift).int()
+
+
+def recall_at(ids, gt):
+    k = gt.shape[1]
+    hit = (ids[:, :, None] == gt[:, None, :]).any(2).sum()
+    return float(hit) / (k * gt.shape[0])
+
+
+def run_ours(args):
+    import torch
+    import torch.distributed as dist
+    import paper_conf_icde_yuwzqzl22_b200 as g
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1:
+        dist.init_process_group("nccl")
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    cfg = syn.CONFIGS[args.config]
+    k = cfg.k
+
+    X, Q = make_workload(cfg, rank)
+    Xd = torch.from_numpy(X).to(dev)
+    Qd = torch.from_numpy(Q).to(dev)
+    torch.cuda.synchronize()
+
+    # ---- GGraphCon build (timed wall clock on device-resident points)
+    t0 = time.perf_counter()
+    graph = g.build(Xd, metric=cfg.metric, degree=cfg.degree)
+    torch.cuda.synchronize()
+    build_s = time.perf_counter() - t0
+    b_iters, b_comps, b_searches, b_rounds = graph.build_stats
+
+    # ---- l sweep -> smallest l with recall@10 >= target
+    gt = ground_truth(torch, Xd, Qd, k)
+    sweep = []
+    chosen = {}
+    for l in L_SWEEP:
+        ids, _ = g.search(graph, Xd, Qd, k, l)
+        r = recall_at(ids, gt)
+        sweep.append((l, round(r, 5)))
+        for tgt in (0.9, 0.95, 0.99):
+            if r >= tgt and tgt not in chosen:
+                chosen[tgt] = l
+        if r >= 0.99:
+            break
+    l_star = chosen.get(args.target, L_SWEEP[-1])
+    ids, dists, st = g.search(graph, Xd, Qd, k, l_star, stats=True)
+    rec = recall_at(ids, gt)
+    st = st.long()
+    d = cfg.d
+    # algorithmic bytes: query + per iteration the adjacency row
+    # + every computed distance's vector row (incl. the entry and lazy-check
+    # re-computations) + the top-k written
+    alg_bytes = int((4 * d + 4 * cfg.degree * st[:, 0] + 4 * d * st[:, 1]).sum().item()
+                    + 8 * k * Q.shape[0])
+    iters_mean = float(st[:, 0].float().mean())
+
+    # ---- timed steps: device-resident inputs, L2 flushed between steps
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+    stream = torch.cuda.current_stream()
+    out = (torch.empty((Q.shape[0], k), dtype=torch.int32, device=dev),
+           torch.empty((Q.shape[0], k), dtype=torch.float32, device=dev))
+    for _ in range(args.warmup):
+        g.search(graph, Xd, Qd, k, l_star, out=out)
+    torch.cuda.synchronize()
+    launches0 = g.kernel_launches()
+    times = []
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    with ClockSampler(local) as clk:
+        for _ in range(args.steps):
+            flush.zero_()
+            e0 = torch.cuda.Event(enable_timing=True)
+            e1 = torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            g.search(graph, Xd, Qd, k, l_star, out=out)
+            e1.record(stream)
+            e1.synchronize()
+            times.append(e0.elapsed_time(e1))
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    launches = g.kernel_launches() - launches0
+    t_total = sum(times) / 1e3
+    t_max = torch.tensor([t_total], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t_max, op=dist.ReduceOp.MAX)
+    t_total = float(t_max.item())
+    total_queries = Q.shape[0] * args.steps * world
+    qps = total_queries / t_total
+    ms_per_step = t_total / args.steps * 1e3
+    kernel_s = statistics.mean(times) / 1e3
+
+    # ---- end to end through the public API from pinned host buffers
+    Qh = torch.from_numpy(Q).pin_memory()
+    hout = (torch.empty((Q.shape[0], k), dtype=torch.int32).pin_memory(),
+            torch.empty((Q.shape[0], k), dtype=torch.float32).pin_memory())
+    for _ in range(2):
+        g.search_host(graph, Xd, Qh, k, l_star, out=hout)
+    e2e_times = []
+    for _ in range(args.steps):
+        flush.zero_()
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        g.search_host(graph, Xd, Qh, k, l_star, out=hout)
+        e2e_times.append(time.perf_counter() - t0)
+    e2e_t = torch.tensor([sum(e2e_times)], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(e2e_t, op=dist.ReduceOp.MAX)
+    e2e_qps = total_queries / float(e2e_t.item())
+
+    peak, peak_kind = peaks()
+    achieved = alg_bytes / kernel_s / 1e9
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(tp):
+        with open(tp) as f:
+            tr = json.load(f)
+        if tr.get("config") == args.config and tr.get("l") == l_star:
+            traffic = tr.get("dram_bytes_per_launch")
+
+    line = {
+        "metric": "queries/sec at recall@10=0.95",
+        "value": round(qps, 1),
+        "unit": "queries/s",
+        "n_gpus": world,
+        "steps": args.steps,
+        "warmup": args.warmup,
+        "ms_per_step": round(ms_per_step, 4),
+        "higher_is_better": True,
+        "scaling": "weak",
+        "vs_baseline": None,
+        "dtype": "f32",
+        "data": "synthetic",
+        "config": {"workload": f"{args.config}: SIFT1M-shaped {cfg.n}x{cfg.d} L2, NSW degree "
+                               f"{cfg.degree}, {Q.shape[0]} queries/GPU, k={k}",
+                   "l": l_star, "e": l_star, "recall_at_10": round(rec, 5),
+                   "l_for_recall": {str(t): chosen.get(t) for t in (0.9, 0.95, 0.99)},
+                   "l_sweep_recall": sweep, "mean_iterations": round(iters_mean, 2),
+                   "l2": "flushed (256 MiB write) between timed steps",
+                   "parallelism": f"replicated graph, query data-parallel x{world}"},
+        "build_seconds": round(build_s, 4),
+        "build": {"iterations": b_iters, "distance_computations": b_comps,
+                  "searches": b_searches, "rounds": b_rounds,
+                  "alg_GBps": round((4 * d * b_comps + 4 * cfg.degree * b_iters) / build_s / 1e9, 1)},
+        "e2e": {"value": round(e2e_qps, 1), "unit": "queries/s",
+                "h2d_bytes_per_step": int(Q.nbytes), "d2h_bytes_per_step": int(Q.shape[0] * k * 8)},
+        "gpu_launches": int(launches),
+        "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak,
+                     "unit": "GB/s", "frac": round(achieved / peak, 4), "traffic": traffic,
+                     "peak_kind": peak_kind, "alg_bytes_per_launch": alg_bytes,
+                     "kernel": "ganns::search_kernel<1,1,true>"},
+        "clocks": clk.summary(),
+    }
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        line["cpu_baseline"] = cpu_baseline(graph.adjacency(), X, Q, k, l_star, args.cpu_seconds)
+    if rank == 0:
+        s = json.dumps(line)
+        print(s, flush=True)
+        if args.json_out:
+            with open(args.json_out, "w") as f:
+                f.write(s + "\n")
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def cpu_baseline(nbr, X, Q, k, l, seconds):
+    """The oracle's search (plain C, one pthread per host core) on a bounded sample
+    of the same queries and graph.  Returns the cpu_baseline object."""
+    import oracle
+    cores = oracle.ncores()
+    m = 64
+    t0 = time.perf_counter()
+    oracle.search(nbr, X, Q[:m], k, l, threads=cores)
+    dt = time.perf_counter() - t0
+    m2 = int(min(len(Q), max(m, m * seconds / max(dt, 1e-3))))
+    t0 = time.perf_counter()
+    oracle.search(nbr, X, Q[:m2], k, l, threads=cores)
+    dt = time.perf_counter() - t0
+    return {"value": round(m2 / dt, 1), "unit": "queries/s", "cores": cores, "kind": "oracle",
+            "sample": f"first {m2} of the {len(Q)} queries, same graph, l={l}, {dt:.1f} s"}
+
+
+def run_reference(args):
+    """The oracle timed as it stands (CPU, all host cores) -- the reference arm."""
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    import torch
+    import oracle
+    import paper_conf_icde_yuwzqzl22_b200 as g
+    cfg = syn.CONFIGS[args.config]
+    k = cfg.k
+    X, Q = make_workload(cfg, 0)
+    # index set-up (not timed): the graph the GPU arm searches, deterministic
+    Xd = torch.from_numpy(X).cuda()
+    graph = g.build(Xd, metric=cfg.metric, degree=cfg.degree)
+    nbr = graph.adjacency()
+    Qd = torch.from_numpy(Q).cuda()
+    gt = ground_truth(torch, Xd, Qd, k)
+    l_star = L_SWEEP[-1]
+    for l in L_SWEEP:
+        ids, _ = g.search(graph, Xd, Qd, k, l)
+        if recall_at(ids, gt) >= args.target:
+            l_star = l
+            break
+    del Xd, Qd
+    cores = oracle.ncores()
+    per_step = 48
+    for _ in range(args.warmup):
+        oracle.search(nbr, X, Q[:16], k, l_star, threads=cores)
+    t0 = time.perf_counter()
+    oracle.search(nbr, X, Q[:per_step], k, l_star, threads=cores)
+    dt = time.perf_counter() - t0
+    per_step = int(max(cores, min(len(Q), per_step * 6.0 / max(dt, 1e-3))))
+    times = []
+    for s in range(args.steps):
+        a = (s * per_step) % max(1, len(Q) - per_step)
+        t0 = time.perf_counter()
+        oracle.search(nbr, X, Q[a:a + per_step], k, l_star, threads=cores)
+        times.append(time.perf_counter() - t0)
+    tot = sum(times)
+    v = per_step * args.steps / tot
+    sample = f"{per_step} queries/step of the {len(Q)}-query batch, same graph, l={l_star}"
+    print(json.dumps({
+        "impl": "reference", "metric": "queries/sec at recall@10=0.95", "value": round(v, 1),
+        "unit": "queries/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": round(tot / args.steps * 1e3, 3), "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+        "config": {"workload": f"{args.config}: SIFT1M-shaped {cfg.n}x{cfg.d} L2, NSW degree "
+                               f"{cfg.degree}, k={k}", "l": l_star},
+        "cpu_baseline": {"value": round(v, 1), "unit": "queries/s", "cores": cores,
+                         "kind": "oracle", "sample": sample},
+        "e2e": {"value": round(v, 1), "unit": "queries/s", "h2d_bytes_per_step": 0,
+                "d2h_bytes_per_step": 0},
+    }), flush=True)
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_ours(args)
+
+
+if __name__ == "__main__":
+    main()
