@@ -44,6 +44,8 @@ def parse():
     ap.add_argument("--config", default="C2")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--target", type=float, default=0.95)
+    ap.add_argument("--l-build", type=int, default=128,
+                    help="candidate-list length of the build searches (P:222: 32/64/128)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
     ap.add_argument("--json-out", default=None)
@@ -60,58 +62,56 @@ def peaks():
 
 
 class ClockSampler:
-    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+    """SM clock + throttle reasons sampled through NVML every ~2 ms while the timed
+    region runs (the recipe's nvidia-smi clocks line, at a rate that resolves a
+    region of tens of milliseconds)."""
 
-    Q = ("index,clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,"
-         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
-         "clocks_event_reasons.sw_power_cap")
+    REASONS = {"hw_slowdown": 0x8, "sw_thermal_slowdown": 0x20, "hw_thermal_slowdown": 0x40,
+               "sw_power_cap": 0x4}
 
     def __init__(self, index: int):
         self.index = index
-        self.proc = None
-        self.lines = []
+        self.samples = []
+        self.stop = threading.Event()
+        self.max_mhz = None
+
+    def _run(self):
+        import pynvml as nv
+        h = nv.nvmlDeviceGetHandleByIndex(self.index)
+        self.max_mhz = float(nv.nvmlDeviceGetMaxClockInfo(h, nv.NVML_CLOCK_SM))
+        while not self.stop.is_set():
+            try:
+                sm = float(nv.nvmlDeviceGetClockInfo(h, nv.NVML_CLOCK_SM))
+                rs = int(nv.nvmlDeviceGetCurrentClocksEventReasons(h))
+            except Exception:
+                break
+            self.samples.append((sm, rs))
+            time.sleep(0.002)
 
     def __enter__(self):
         try:
-            self.proc = subprocess.Popen(
-                ["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.Q}",
-                 "--format=csv,noheader,nounits", "-lms", "100"],
-                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
-            self.t = threading.Thread(target=self._read, daemon=True)
+            import pynvml as nv
+            nv.nvmlInit()
+            vis = os.environ.get("CUDA_VISIBLE_DEVICES")
+            if vis:
+                self.index = int(vis.split(",")[self.index])
+            self.t = threading.Thread(target=self._run, daemon=True)
             self.t.start()
-        except FileNotFoundError:
-            self.proc = None
+            time.sleep(0.01)
+        except Exception:
+            self.t = None
         return self
 
-    def _read(self):
-        for line in self.proc.stdout:
-            self.lines.append(line.strip())
-
     def __exit__(self, *a):
-        if self.proc:
-            self.proc.terminate()
-            try:
-                self.proc.wait(timeout=5)
-            except subprocess.TimeoutExpired:
-                self.proc.kill()
+        self.stop.set()
+        if self.t:
+            self.t.join(timeout=2)
 
     def summary(self):
-        sm, mx, reasons = [], None, set()
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        for ln in self.lines:
-            f = [x.strip() for x in ln.split(",")]
-            if len(f) < 7:
-                continue
-            try:
-                sm.append(float(f[1]))
-                mx = float(f[2])
-            except ValueError:
-                continue
-            for nm, v in zip(names, f[3:7]):
-                if v.lower().startswith("active"):
-                    reasons.add(nm)
-        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": mx,
-                "reasons": sorted(reasons), "samples": len(sm)}
+        sm = [s for s, _ in self.samples]
+        reasons = sorted({n for _, r in self.samples for n, bit in self.REASONS.items() if r & bit})
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": self.max_mhz,
+                "reasons": reasons, "samples": len(sm)}
 
 
 def make_workload(cfg, rank: int):
@@ -169,7 +169,7 @@ def run_ours(args):
 
     # ---- GGraphCon build (timed wall clock on device-resident points)
     t0 = time.perf_counter()
-    graph = g.build(Xd, metric=cfg.metric, degree=cfg.degree)
+    graph = g.build(Xd, metric=cfg.metric, degree=cfg.degree, l_build=args.l_build)
     torch.cuda.synchronize()
     build_s = time.perf_counter() - t0
     b_iters, b_comps, b_searches, b_rounds = graph.build_stats
@@ -285,6 +285,8 @@ def run_ours(args):
                    "l2": "flushed (256 MiB write) between timed steps",
                    "parallelism": f"replicated graph, query data-parallel x{world}"},
         "build_seconds": round(build_s, 4),
+        "build_params": {"degree": cfg.degree, "d_min": cfg.degree // 2, "l_build": args.l_build,
+                         "group_size": "auto"},
         "build": {"iterations": b_iters, "distance_computations": b_comps,
                   "searches": b_searches, "rounds": b_rounds,
                   "alg_GBps": round((4 * d * b_comps + 4 * cfg.degree * b_iters) / build_s / 1e9, 1)},
@@ -340,7 +342,7 @@ def run_reference(args):
     X, Q = make_workload(cfg, 0)
     # index set-up (not timed): the graph the GPU arm searches, deterministic
     Xd = torch.from_numpy(X).cuda()
-    graph = g.build(Xd, metric=cfg.metric, degree=cfg.degree)
+    graph = g.build(Xd, metric=cfg.metric, degree=cfg.degree, l_build=args.l_build)
     nbr = graph.adjacency()
     Qd = torch.from_numpy(Q).cuda()
     gt = ground_truth(torch, Xd, Qd, k)

@@ -16,7 +16,7 @@ import numpy as np
 import torch
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libganns.so")
+LIB_PATH = os.environ.get("GANNS_LIB_PATH") or os.path.join(_HERE, "libganns.so")
 
 METRICS = {"l2": 0, "ip": 1, "cosine": 2}
 _METRIC_NAMES = {v: k for k, v in METRICS.items()}

@@ -18,12 +18,24 @@ OBJ = os.path.join(PKG, "_obj")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-fvisibility=hidden",
-         "-I", os.path.join(ROOT, "include")]
+         "-I", os.path.join(ROOT, "include")] + os.environ.get("GANNS_NVCC_EXTRA", "").split()
 
 # (source, extra defines, object name)
 UNITS = [("api.cu", [], "api.o"), ("search.cu", [], "search.o")] + \
         [("search_inst.cu", [f"-DGANNS_NV4={v}"], f"search_nv{v}.o") for v in (1, 2, 4, 8)] + \
         [("build_inst.cu", [f"-DGANNS_NV4={v}"], f"build_nv{v}.o") for v in (1, 2, 4, 8)]
+# GANNS_DEV=1: developer flavour with only the d <= 128 / d_max <= 32 / L2
+# instances (fast rebuilds while tuning).  Never shipped: the flavour stamp
+# makes build() rebuild the full library.
+DEV_UNITS = [("api.cu", ["-DGANNS_DEV_NV1"], "dev_api.o"),
+             ("search.cu", ["-DGANNS_DEV_NV1"], "dev_search.o"),
+             ("search_inst.cu", ["-DGANNS_NV4=1", "-DGANNS_DEV_ONE"], "dev_search_nv1.o"),
+             ("build_inst.cu", ["-DGANNS_NV4=1", "-DGANNS_DEV_ONE"], "dev_build_nv1.o")]
+FLAVOR = os.path.join(PKG, "libganns.flavor")
+
+
+def _flavor():
+    return "dev" if os.environ.get("GANNS_DEV") == "1" else "full"
 
 
 def _sources():
@@ -33,6 +45,8 @@ def _sources():
 
 def stale() -> bool:
     if not os.path.exists(LIB):
+        return True
+    if not os.path.exists(FLAVOR) or open(FLAVOR).read().strip() != _flavor():
         return True
     t = os.path.getmtime(LIB)
     return any(os.path.getmtime(s) > t for s in _sources())
@@ -52,14 +66,17 @@ def build(force: bool = False, verbose: bool = False) -> str:
     if not force and not stale():
         return LIB
     os.makedirs(OBJ, exist_ok=True)
-    with cf.ThreadPoolExecutor(max_workers=max(2, min(len(UNITS), os.cpu_count() or 2))) as ex:
-        objs = list(ex.map(_compile, UNITS))
+    units = DEV_UNITS if _flavor() == "dev" else UNITS
+    with cf.ThreadPoolExecutor(max_workers=max(2, min(len(units), os.cpu_count() or 2))) as ex:
+        objs = list(ex.map(_compile, units))
     tmp = LIB + f".{os.getpid()}.tmp"
     cmd = [NVCC, *ARCH, "-shared", "-o", tmp, *objs, "-lcudart"]
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         raise RuntimeError(f"link failed:\n{r.stderr}")
     os.replace(tmp, LIB)
+    with open(FLAVOR, "w") as f:
+        f.write(_flavor())
     if verbose:
         print("built", LIB)
     return LIB

@@ -48,12 +48,36 @@ struct HostPipe {
 static std::mutex g_pipe_mu;
 static HostPipe g_pipes[64];
 
+// Ticket counters for the persistent search kernel: a ring of device ints per
+// device, one slot per launch (concurrent launches on different streams get
+// different slots; 4096 launches would have to be in flight to wrap).
+constexpr int kTicketSlots = 4096;
+static std::mutex g_ticket_mu;
+static int32_t* g_tickets[64] = {nullptr};
+static std::atomic<uint32_t> g_ticket_next{0};
+
+int32_t* ticket_slot() {
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (dev < 0 || dev >= 64) return nullptr;
+  {
+    std::lock_guard<std::mutex> lock(g_ticket_mu);
+    if (!g_tickets[dev] && cudaMalloc(&g_tickets[dev], sizeof(int32_t) * kTicketSlots) != cudaSuccess) {
+      g_tickets[dev] = nullptr;
+      return nullptr;
+    }
+  }
+  return g_tickets[dev] + (g_ticket_next.fetch_add(1) % kTicketSlots);
+}
+
 int run_build(BuildArgs& a, cudaStream_t s) {
   switch (nv4_for(a.d)) {
     case 1: return run_build_nv<1>(a, s);
+#ifndef GANNS_DEV_NV1
     case 2: return run_build_nv<2>(a, s);
     case 4: return run_build_nv<4>(a, s);
     case 8: return run_build_nv<8>(a, s);
+#endif
   }
   return fail(GANNS_ENOTSUP, "unsupported dimension");
 }
@@ -200,7 +224,7 @@ static int validate_search(const ganns_graph* g, const float* points, const floa
                            const void* out_ids, const void* out_dists, int* e_out,
                            int32_t* entry_out) {
   if (int rc = check_graph(g)) return rc;
-  if (nq < 0) return fail(GANNS_EINVAL, "nq < 0");
+  if (nq < 0 || nq >= (int64_t(1) << 31)) return fail(GANNS_EINVAL, "nq must be in [0, 2^31)");
   if (k < 1 || k >= g->n) return fail(GANNS_EINVAL, "k must be in [1, n)");
   if (l < k || l > 1024) return fail(GANNS_EINVAL, "l must be in [k, 1024]");
   int e = p ? p->e : 0;
@@ -223,8 +247,10 @@ int ganns_search_ex(const ganns_graph* g, const float* points, const float* quer
   if (int rc = validate_search(g, points, queries, nq, k, l, p, out_ids, out_dists, &e, &entry))
     return rc;
   if (nq == 0) return GANNS_OK;
+  int32_t* tk = ticket_slot();
+  if (!tk) return fail(GANNS_ENOMEM, "ticket allocation failed");
   SearchLaunch a{g->nbr, points, g->n, g->d, g->d_max, g->metric, queries, nq, k, l, e, entry,
-                 out_ids, out_dists, p ? p->stats : nullptr};
+                 out_ids, out_dists, p ? p->stats : nullptr, tk};
   cudaError_t err = launch_search(a, static_cast<cudaStream_t>(stream));
   return err == cudaSuccess ? GANNS_OK : cuda_fail(err, "search kernel launch");
 }
@@ -291,8 +317,10 @@ int ganns_search_host(const ganns_graph* g, const float* points, const float* qu
     err = cudaMemcpyAsync(P.dq[b], queries_host + size_t(q0) * g->d, sizeof(float) * m * g->d,
                           cudaMemcpyHostToDevice, s);
     if (err != cudaSuccess) break;
+    int32_t* tk = ticket_slot();
+    if (!tk) return fail(GANNS_ENOMEM, "ticket allocation failed");
     SearchLaunch a{g->nbr, points, g->n, g->d, g->d_max, g->metric, P.dq[b], m, k, l, e, entry,
-                   P.dids[b], P.ddst[b], nullptr};
+                   P.dids[b], P.ddst[b], nullptr, tk};
     err = launch_search(a, s);
     if (err != cudaSuccess) break;
     err = cudaMemcpyAsync(out_ids_host + size_t(q0) * k, P.dids[b], sizeof(int32_t) * m * k,

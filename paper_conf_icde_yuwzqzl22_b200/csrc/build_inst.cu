@@ -121,10 +121,11 @@ phase1_kernel(BuildDev B, int64_t group_size, int64_t ngroups) {
   const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int64_t gi = int64_t(blockIdx.x) * kBuildWarps + w;
   if (gi >= ngroups) return;
-  uint8_t* base = smem + size_t(w) * warp_smem_bytes(B.l_build, TPL);
-  uint64_t* sN = reinterpret_cast<uint64_t*>(base);
-  uint64_t* sT = sN + lpad32(B.l_build);
-  uint32_t* sBM = reinterpret_cast<uint32_t*>(sT + TPL * 32);
+  WarpSmem ws = carve_warp_smem(smem + size_t(w) * warp_smem_bytes(B.l_build, TPL, NV4, B.g.d4),
+                                B.l_build, TPL, NV4, B.g.d4);
+  if (lane == 0) mbar_init(ws.mbar, 1);
+  __syncwarp();
+  uint64_t* sN = ws.sN;
   const int64_t lo = gi * group_size;
   const int64_t hi = lo + group_size < B.g.n ? lo + group_size : B.g.n;
   const int d = B.g.d4 * 4;
@@ -132,7 +133,7 @@ phase1_kernel(BuildDev B, int64_t group_size, int64_t ngroups) {
     // Step 1 (line 5): v.N, v.N' := Search(G_i, v, d_min), entry = group's first vertex
     SearchStats st;
     const int cnt = warp_search<NV4, TPL, L2, true>(B.g, B.g.X + size_t(v) * d, int32_t(lo),
-                                                    B.l_build, B.e_build, sN, sT, sBM, st);
+                                                    B.l_build, B.e_build, ws, st);
     add_stats(B.stats, st, lane);
     const int m = cnt < B.d_min ? cnt : B.d_min;
     for (int j = lane; j < m; j += 32) {
@@ -167,15 +168,17 @@ round_search_kernel(BuildDev B, int64_t lo, int64_t hi, int32_t* __restrict__ Eu
   const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int64_t v = lo + int64_t(blockIdx.x) * kBuildWarps + w;
   if (v >= hi) return;
-  uint8_t* base = smem + size_t(w) * warp_smem_bytes(B.l_build, TPL);
-  uint64_t* sN = reinterpret_cast<uint64_t*>(base);
-  uint64_t* sT = sN + lpad32(B.l_build);
-  uint32_t* sBM = reinterpret_cast<uint32_t*>(sT + TPL * 32);
+  WarpSmem ws = carve_warp_smem(smem + size_t(w) * warp_smem_bytes(B.l_build, TPL, NV4, B.g.d4),
+                                B.l_build, TPL, NV4, B.g.d4);
+  if (lane == 0) mbar_init(ws.mbar, 1);
+  __syncwarp();
+  uint64_t* sN = ws.sN;
+  uint64_t* sT = ws.sT;
   const int d = B.g.d4 * 4;
   // line 12: v.N := Search(G_0, v, d_min); G_0 = P_0..P_{i-1}, entry = vertex 0
   SearchStats st;
   const int cnt = warp_search<NV4, TPL, L2, false>(B.g, B.g.X + size_t(v) * d, 0, B.l_build,
-                                                   B.e_build, sN, sT, sBM, st);
+                                                   B.e_build, ws, st);
   add_stats(B.stats, st, lane);
   const int dm = B.d_min;
   const int cs = cnt < dm ? cnt : dm;
@@ -296,7 +299,7 @@ template <int NV4, int TPL, bool L2>
 static cudaError_t set_smem_attrs() {
   static bool done = false;
   if (done) return cudaSuccess;
-  const int mx = int(kBuildWarps * warp_smem_bytes(1024, TPL));
+  const int mx = 227 * 1024;
   cudaError_t e = cudaFuncSetAttribute(phase1_kernel<NV4, TPL, L2>,
                                        cudaFuncAttributeMaxDynamicSharedMemorySize, mx);
   if (e == cudaSuccess)
@@ -367,7 +370,8 @@ static int build_t(BuildArgs& a, cudaStream_t s) {
   B.l_build = a.l_build;
   B.e_build = a.e_build;
   B.stats = stats.p;
-  const size_t smem = size_t(kBuildWarps) * warp_smem_bytes(a.l_build, TPL);
+  const size_t smem = size_t(kBuildWarps) * warp_smem_bytes(a.l_build, TPL, NV4, a.d / 4);
+  if (smem > 227 * 1024) return fail(-4, "build: shared memory per CTA exceeds 227 KB");
 
   // Phase 1 (lines 2-8): all local graphs in parallel, one warp per group
   phase1_kernel<NV4, TPL, L2><<<unsigned((ngroups + kBuildWarps - 1) / kBuildWarps),
@@ -408,10 +412,16 @@ static int build_t(BuildArgs& a, cudaStream_t s) {
 
 template <int NV4, int TPL>
 static int build_m(BuildArgs& a, cudaStream_t s) {
+#ifdef GANNS_DEV_ONE
+  return build_t<NV4, TPL, true>(a, s);
+#endif
   return a.metric == 0 ? build_t<NV4, TPL, true>(a, s) : build_t<NV4, TPL, false>(a, s);
 }
 template <int NV4>
 int run_build_nv(BuildArgs& a, cudaStream_t s) {
+#ifdef GANNS_DEV_ONE
+  return build_m<NV4, 1>(a, s);
+#endif
   switch (tpl_for(a.d_max)) {
     case 1: return build_m<NV4, 1>(a, s);
     case 2: return build_m<NV4, 2>(a, s);

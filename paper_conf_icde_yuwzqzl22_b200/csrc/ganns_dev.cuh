@@ -70,6 +70,52 @@ __device__ __forceinline__ float4 ldg_stream(const float4* p) {
                : "=f"(r.x), "=f"(r.y), "=f"(r.z), "=f"(r.w) : "l"(p));
   return r;
 }
+// Bulk L2 prefetch of one vector row (TMA unit, no registers held): issued for
+// every neighbour as soon as the adjacency row arrives, so the register-staged
+// loads of the bulk-distance passes find their lines in L2.
+__device__ __forceinline__ void prefetch_row_l2(const void* p, uint32_t bytes) {
+  asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p), "r"(bytes) : "memory");
+}
+// ---- TMA (cp.async.bulk) + mbarrier helpers (sm_90+; SASS UBLKCP / SYNCS)
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return uint32_t(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint64_t* m, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(m)), "r"(count) : "memory");
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* m, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(m)), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* m, uint32_t phase) {
+  uint32_t done = 0;
+  do {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+        "selp.u32 %0, 1, 0, p;\n\t}"
+        : "=r"(done) : "r"(smem_u32(m)), "r"(phase) : "memory");
+  } while (!done);
+}
+// 1-D bulk copy global -> shared, completion counted on mbarrier m (bytes % 16 == 0)
+__device__ __forceinline__ void tma_row(void* dst, const void* src, uint32_t bytes, uint64_t* m) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(m))
+      : "memory");
+}
+// Shared-memory 128-bit load kept in program order (bounds register pressure:
+// ptxas may not hoist all passes' loads of a round ahead of their math).
+__device__ __forceinline__ float4 lds128_ordered(const float4* p) {
+  float4 r;
+  asm volatile("ld.volatile.shared.v4.f32 {%0,%1,%2,%3}, [%4];"
+               : "=f"(r.x), "=f"(r.y), "=f"(r.z), "=f"(r.w) : "r"(smem_u32(p)));
+  return r;
+}
+__device__ __forceinline__ void fence_proxy_async_smem() {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+
 template <bool COHERENT>
 __device__ __forceinline__ int32_t load_nbr(const int32_t* p) {
   if constexpr (COHERENT) return *reinterpret_cast<const volatile int32_t*>(p);
@@ -91,50 +137,178 @@ struct SearchStats {
   uint32_t iters, comps, merged;
 };
 
-// Distances of the <= 32 rows in one T slot group, lane j -> delta(q, row of u_j).
-// NV4 = float4 per lane per row (ceil(d/128)); B rows per batch.
-template <int NV4, bool L2>
-__device__ __forceinline__ float group_distances(const GraphView& g, const float4 (&qv)[NV4],
-                                                 int32_t u_mine, float cbase, float qinv,
-                                                 int lane) {
-  constexpr int B = NV4 >= 8 ? 1 : 8 / NV4;
+// Per-warp shared memory: [stage: 32 vector rows, TMA destination][N][T][mbar][bitmap]
+__host__ __device__ constexpr int lpad32(int l) { return (l + 31) & ~31; }
+__host__ __device__ constexpr bool uses_tma(int nv4) { return nv4 <= 2; }
+#ifndef GANNS_STAGE_ROUNDS
+#define GANNS_STAGE_ROUNDS 2
+#endif
+constexpr int kStageRounds = GANNS_STAGE_ROUNDS;   // rows are staged in kStageRounds TMA rounds
+constexpr int kStageRows = 32 / kStageRounds;
+__host__ __device__ constexpr size_t stage_bytes(int nv4, int d4) {
+  return uses_tma(nv4) ? size_t(kStageRows) * d4 * 16 : 0;
+}
+__host__ __device__ constexpr size_t warp_smem_bytes(int l, int tpl, int nv4, int d4) {
+  return stage_bytes(nv4, d4) + size_t(lpad32(l)) * 8 + size_t(tpl) * 32 * 8 + 16 + 128;
+}
+struct WarpSmem {
+  float4* stage;
+  uint64_t* sN;
+  uint64_t* sT;
+  uint64_t* mbar;
+  uint32_t* sBM;
+  uint32_t phase;   // parity of the next mbarrier phase to wait for
+};
+__device__ __forceinline__ WarpSmem carve_warp_smem(uint8_t* base, int l, int tpl, int nv4, int d4) {
+  WarpSmem w;
+  w.stage = reinterpret_cast<float4*>(base);
+  w.sN = reinterpret_cast<uint64_t*>(base + stage_bytes(nv4, d4));
+  w.sT = w.sN + lpad32(l);
+  w.mbar = w.sT + tpl * 32;
+  w.sBM = reinterpret_cast<uint32_t*>(w.mbar + 2);
+  w.phase = 0;
+  return w;
+}
+
+// Vector layout per dimension bucket (NV4 = template selector, see nv4_for):
+// S lanes share one row, each lane owning C float4 columns (i4 = lane%S + S*f).
+// d <= 128: 8 lanes x 4 float4 per row, so one warp-wide 128-bit load covers 4
+// rows (each 128 B-coalesced) and 8 rows are in flight per lane per group pass.
+template <int NV4> struct VecLayout;
+template <> struct VecLayout<1> { static constexpr int S = 8, C = 4; };    // d <= 128
+template <> struct VecLayout<2> { static constexpr int S = 16, C = 4; };   // d <= 256
+template <> struct VecLayout<4> { static constexpr int S = 32, C = 4; };   // d <= 512
+template <> struct VecLayout<8> { static constexpr int S = 32, C = 8; };   // d <= 1024
+
+// Packed fp32x2 arithmetic (sm_100a FADD2 / FFMA2): one instruction per two
+// lanes of a float4, halving the FP instruction count of the bulk distance.
+// The two halves are summed at the end (the order of an fp32 sum; exact on the
+// integer-grid inputs, R-C18).
+__device__ __forceinline__ uint64_t pk2(float a, float b) {
+  uint64_t r;
+  asm("mov.b64 %0, {%1,%2};" : "=l"(r) : "f"(a), "f"(b));
+  return r;
+}
+__device__ __forceinline__ float hsum2(uint64_t v) {
+  float lo, hi;
+  asm("mov.b64 {%0,%1}, %2;" : "=f"(lo), "=f"(hi) : "l"(v));
+  return lo + hi;
+}
+template <bool L2>
+__device__ __forceinline__ uint64_t accum4(uint64_t acc, const float4& q, const float4& x) {
+  const uint64_t qa = pk2(q.x, q.y), qb = pk2(q.z, q.w);
+  const uint64_t xa = pk2(x.x, x.y), xb = pk2(x.z, x.w);
+  if constexpr (L2) {
+    uint64_t ta, tb;
+    asm("sub.rn.f32x2 %0, %1, %2;" : "=l"(ta) : "l"(qa), "l"(xa));
+    asm("sub.rn.f32x2 %0, %1, %2;" : "=l"(tb) : "l"(qb), "l"(xb));
+    asm("fma.rn.f32x2 %0, %1, %1, %0;" : "+l"(acc) : "l"(ta));
+    asm("fma.rn.f32x2 %0, %1, %1, %0;" : "+l"(acc) : "l"(tb));
+  } else {
+    asm("fma.rn.f32x2 %0, %1, %2, %0;" : "+l"(acc) : "l"(qa), "l"(xa));
+    asm("fma.rn.f32x2 %0, %1, %2, %0;" : "+l"(acc) : "l"(qb), "l"(xb));
+  }
+  return acc;
+}
+
+// Bulk distance for the <= 32 neighbours held one per lane (u_mine,
+// -1 = none): returns, in lane j, the raw sum for u_j (L2: squared distance,
+// IP/COSINE: dot product).
+// Math layout: S-lane segments; in pass g segment s works on the row of lane
+// g + S*s (its 8 lanes read 128 B contiguous from shared memory, conflict-free);
+// after S passes a transposing butterfly inside the segment leaves lane j with
+// row j's total.
+// Gather: the rows of the passes of one round are fetched by TMA bulk copies
+// (one cp.async.bulk per lane that owns a row of the round) into the warp's
+// stage buffer and waited for with a single mbarrier phase -- kStageRounds
+// memory round trips per iteration, no registers held in flight.
+template <int S, int C, bool L2, bool FULL>
+__device__ __forceinline__ float tma_dot(const GraphView& g, const float4 (&qv)[C],
+                                         int32_t u_mine, int lane, WarpSmem& ws) {
+  static_assert(S % kStageRounds == 0, "passes must split evenly into rounds");
+  constexpr int PPR = S / kStageRounds;             // passes per round
+  const int sl = lane & (S - 1), seg = lane / S;
+  const uint32_t rowbytes = uint32_t(g.d4) * 16u;
+  // lane j = g + S*s holds the row of pass g of segment s; it is staged in round
+  // g / PPR at slot (g % PPR) + PPR*s
+  const int my_round = sl / PPR;
+  const int my_slot = sl % PPR + PPR * seg;
+  int coff[C];
+#pragma unroll
+  for (int f = 0; f < C; ++f) coff[f] = (FULL || sl + S * f < g.d4) ? sl + S * f : g.d4 - 1;
+  float p[S];
+#pragma unroll
+  for (int r = 0; r < kStageRounds; ++r) {
+    const bool mine = u_mine >= 0 && my_round == r;
+    const unsigned vm = __ballot_sync(kFull, mine);
+    if (vm) {
+      __syncwarp();
+      fence_proxy_async_smem();   // earlier generic reads of the stage precede the async writes
+      if (lane == 0) mbar_arrive_expect_tx(ws.mbar, uint32_t(__popc(vm)) * rowbytes);
+      __syncwarp();
+      if (mine)
+        tma_row(reinterpret_cast<char*>(ws.stage) + size_t(my_slot) * rowbytes,
+                reinterpret_cast<const char*>(g.X) + uint64_t(uint32_t(u_mine)) * rowbytes,
+                rowbytes, ws.mbar);
+      mbar_wait(ws.mbar, ws.phase);
+      ws.phase ^= 1u;
+    }
+#pragma unroll
+    for (int gg = 0; gg < PPR; ++gg) {
+      const float4* rp = ws.stage + size_t(gg + PPR * seg) * g.d4;
+      float4 x[C];
+#pragma unroll
+      for (int f = 0; f < C; ++f) x[f] = lds128_ordered(rp + coff[f]);
+      uint64_t acc = 0;
+#pragma unroll
+      for (int f = 0; f < C; ++f)
+        if (FULL || sl + S * f < g.d4) acc = accum4<L2>(acc, qv[f], x[f]);
+      p[r * PPR + gg] = hsum2(acc);
+    }
+  }
+#pragma unroll
+  for (int half = S / 2; half >= 1; half >>= 1) {
+    const bool up = lane & half;
+#pragma unroll
+    for (int i = 0; i < half; ++i) {
+      float send = up ? p[i] : p[i + half];
+      float keep = up ? p[i + half] : p[i];
+      p[i] = keep + __shfl_xor_sync(kFull, send, half);
+    }
+  }
+  return p[0];
+}
+
+// Whole-warp form (S = 32, d > 256): rows in batches of B, a transposing
+// butterfly over the top log2(B) lane bits, plain reduction over the rest.
+template <int C, bool L2, bool FULL>
+__device__ __forceinline__ float warp_dot(const GraphView& g, const float4 (&qv)[C],
+                                          int32_t u_mine, int lane) {
+  constexpr int B = C >= 8 ? 1 : 8 / C;
   constexpr int LOGB = B == 8 ? 3 : B == 4 ? 2 : B == 2 ? 1 : 0;
-  const float4* X4 = reinterpret_cast<const float4*>(g.X);
+  const char* base = reinterpret_cast<const char*>(g.X) + lane * 16;
+  const uint32_t rowbytes = uint32_t(g.d4) * 16u;
+  const int32_t u_safe = u_mine < 0 ? 0 : u_mine;
+  int coff[C];
+#pragma unroll
+  for (int f = 0; f < C; ++f) coff[f] = (FULL || lane + 32 * f < g.d4) ? 32 * f : g.d4 - 1 - lane;
   float dres = 0.f;
 #pragma unroll
   for (int b = 0; b < 32 / B; ++b) {
-    float4 buf[B][NV4];
-    int32_t ub[B];
-#pragma unroll
-    for (int i = 0; i < B; ++i) {
-      ub[i] = __shfl_sync(kFull, u_mine, b * B + i);
-      const float4* row = X4 + size_t(ub[i] < 0 ? 0 : ub[i]) * g.d4;
-#pragma unroll
-      for (int f = 0; f < NV4; ++f) {
-        int i4 = lane + 32 * f;
-        buf[i][f] = (ub[i] >= 0 && i4 < g.d4) ? ldg_stream(row + i4) : make_float4(0.f, 0.f, 0.f, 0.f);
-      }
-    }
     float p[B];
 #pragma unroll
     for (int i = 0; i < B; ++i) {
-      float acc = 0.f;
+      const int32_t u = __shfl_sync(kFull, u_safe, b * B + i);
+      const float4* rp = reinterpret_cast<const float4*>(base + uint64_t(uint32_t(u)) * rowbytes);
+      float4 x[C];
 #pragma unroll
-      for (int f = 0; f < NV4; ++f) {
-        const float4 x = buf[i][f], q = qv[f];
-        if constexpr (L2) {
-          float t0 = q.x - x.x, t1 = q.y - x.y, t2 = q.z - x.z, t3 = q.w - x.w;
-          acc = fmaf(t0, t0, acc); acc = fmaf(t1, t1, acc);
-          acc = fmaf(t2, t2, acc); acc = fmaf(t3, t3, acc);
-        } else {
-          acc = fmaf(q.x, x.x, acc); acc = fmaf(q.y, x.y, acc);
-          acc = fmaf(q.z, x.z, acc); acc = fmaf(q.w, x.w, acc);
-        }
-      }
-      p[i] = acc;
+      for (int f = 0; f < C; ++f) x[f] = ldg_stream(rp + coff[f]);
+      uint64_t acc = 0;
+#pragma unroll
+      for (int f = 0; f < C; ++f)
+        if (FULL || lane + 32 * f < g.d4) acc = accum4<L2>(acc, qv[f], x[f]);
+      p[i] = hsum2(acc);
     }
-    // transposing butterfly: after LOGB stages lane L holds batch entry
-    // (L >> (5-LOGB)) summed over the lanes that differ in the top LOGB bits
 #pragma unroll
     for (int s = 0; s < LOGB; ++s) {
       const int half = B >> (s + 1), off = 16 >> s;
@@ -151,42 +325,60 @@ __device__ __forceinline__ float group_distances(const GraphView& g, const float
     float got = __shfl_sync(kFull, p[0], (lane & (B - 1)) << (5 - LOGB));
     if ((lane >> LOGB) == b) dres = got;
   }
-  if constexpr (L2) return dres;
-  else return cbase - dres * qinv;   // IP: 0 - dot (exact); COSINE: 1 - dot/||q||
+  return dres;
 }
 
-// Shared-memory footprint of one warp's search state for list length l.
-__host__ __device__ constexpr int lpad32(int l) { return (l + 31) & ~31; }
-__host__ __device__ constexpr size_t warp_smem_bytes(int l, int tpl) {
-  return size_t(lpad32(l)) * 8 + size_t(tpl) * 32 * 8 + 32 * 4;
+template <int NV4, bool L2>
+__device__ __forceinline__ float group_distances(const GraphView& g,
+                                                 const float4 (&qv)[VecLayout<NV4>::C],
+                                                 int32_t u_mine, float cbase, float qinv,
+                                                 int lane, WarpSmem& ws) {
+  constexpr int S = VecLayout<NV4>::S, C = VecLayout<NV4>::C;
+  static_assert(uses_tma(NV4) == (S < 32), "TMA staging is used exactly for the segment form");
+  const bool full = g.d4 == S * C;
+  float dot;
+  if constexpr (S < 32) {
+    dot = full ? tma_dot<S, C, L2, true>(g, qv, u_mine, lane, ws)
+               : tma_dot<S, C, L2, false>(g, qv, u_mine, lane, ws);
+  } else {
+    dot = full ? warp_dot<C, L2, true>(g, qv, u_mine, lane)
+               : warp_dot<C, L2, false>(g, qv, u_mine, lane);
+  }
+  if constexpr (L2) return dot;
+  else return cbase - dot * qinv;   // IP: 0 - dot (exact); COSINE: 1 - dot/||q||
 }
+
 
 // The GANNS search of one query by one warp.  On return sN[0..cnt) holds N
 // (ascending, explored flags set); returns cnt.  COHERENT: read the graph with
 // coherent loads (the build modifies it inside the same kernel).
 template <int NV4, int TPL, bool L2, bool COHERENT>
 __device__ int warp_search(const GraphView& g, const float* __restrict__ qrow, int32_t entry,
-                           int l, int e, uint64_t* sN, uint64_t* sT, uint32_t* sBM,
-                           SearchStats& st) {
+                           int l, int e, WarpSmem& ws, SearchStats& st) {
   const int lane = threadIdx.x & 31;
+  uint64_t* sN = ws.sN;
+  uint64_t* sT = ws.sT;
+  uint32_t* sBM = ws.sBM;
   const int lp = lpad32(l);
   const int nwords = lp >> 5;
-  // query slice in registers
-  float4 qv[NV4];
+  // query slice in registers: lane owns float4 columns
+  // lane%S + S*f (every S-lane segment holds a full copy of q)
+  constexpr int S = VecLayout<NV4>::S, C = VecLayout<NV4>::C;
+  float4 qv[C];
   const float4* q4 = reinterpret_cast<const float4*>(qrow);
 #pragma unroll
-  for (int f = 0; f < NV4; ++f) {
-    int i4 = lane + 32 * f;
+  for (int f = 0; f < C; ++f) {
+    int i4 = (lane & (S - 1)) + S * f;
     qv[f] = i4 < g.d4 ? q4[i4] : make_float4(0.f, 0.f, 0.f, 0.f);
   }
   float cbase = 0.f, qinv = 1.f;
   if (!L2 && g.metric == 2) {
     float s = 0.f;
 #pragma unroll
-    for (int f = 0; f < NV4; ++f)
+    for (int f = 0; f < C; ++f)
       s += qv[f].x * qv[f].x + qv[f].y * qv[f].y + qv[f].z * qv[f].z + qv[f].w * qv[f].w;
 #pragma unroll
-    for (int off = 16; off >= 1; off >>= 1) s += __shfl_xor_sync(kFull, s, off);
+    for (int off = S / 2; off >= 1; off >>= 1) s += __shfl_xor_sync(kFull, s, off);
     cbase = 1.f;
     qinv = 1.f / sqrtf(s);
   }
@@ -195,7 +387,7 @@ __device__ int warp_search(const GraphView& g, const float* __restrict__ qrow, i
   if (lane < nwords) sBM[lane] = 0u;
   {
     int32_t u = lane == 0 ? entry : -1;
-    float dd = group_distances<NV4, L2>(g, qv, u, cbase, qinv, lane);
+    float dd = group_distances<NV4, L2>(g, qv, u, cbase, qinv, lane, ws);
     if (lane == 0) sN[0] = mkkey(dd, entry);
   }
   __syncwarp();
@@ -234,10 +426,16 @@ __device__ int warp_search(const GraphView& g, const float* __restrict__ qrow, i
       u[t] = j < g.d_max ? load_nbr<COHERENT>(row + j) : -1;
     }
     // (3) bulk distance computation
+    if constexpr (!uses_tma(NV4)) {
+#pragma unroll
+      for (int t = 0; t < TPL; ++t)
+        if (u[t] >= 0)
+          prefetch_row_l2(g.X + size_t(u[t]) * (g.d4 * 4), uint32_t(g.d4) * 16u);
+    }
     uint64_t key[TPL];
 #pragma unroll
     for (int t = 0; t < TPL; ++t) {
-      float dd = group_distances<NV4, L2>(g, qv, u[t], cbase, qinv, lane);
+      float dd = group_distances<NV4, L2>(g, qv, u[t], cbase, qinv, lane, ws);
       key[t] = u[t] >= 0 ? mkkey(dd, u[t]) : kKeyInf;
       st.comps += __popc(__ballot_sync(kFull, u[t] >= 0));
     }

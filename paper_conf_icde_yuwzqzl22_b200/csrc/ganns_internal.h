@@ -17,7 +17,13 @@ struct ganns_graph {
 
 namespace ganns {
 
-constexpr int kWarpsPerBlock = 4;   // queries (warps) per CTA of the search kernel
+constexpr int kWarpsPerBlock = 4;   // warps per CTA of the small helper kernels
+constexpr int kSearchWarps = 2;     // warps (= concurrent queries) per CTA of the search kernel
+#ifndef GANNS_MIN_BLOCKS
+#define GANNS_MIN_BLOCKS 12
+#endif
+constexpr int kMinBlocksPerSM = GANNS_MIN_BLOCKS; // register budget: <= 85 regs/thread (24 warps per SM);
+                                    // the TMA stage (8 KB/warp at d=128) allows ~22 warps
 
 void set_error(const std::string& msg);
 int fail(int status, const std::string& msg);
@@ -43,7 +49,9 @@ struct SearchLaunch {
   int32_t* out_ids;
   float* out_dists;
   uint32_t* stats;
+  int32_t* ticket;      // device scratch counter for the persistent scheduler
 };
+int32_t* ticket_slot();   // a device int reserved for one launch (ring of slots)
 cudaError_t launch_search(const SearchLaunch& a, cudaStream_t s);
 template <int NV4>
 cudaError_t launch_search_nv(const SearchLaunch& a, cudaStream_t s);

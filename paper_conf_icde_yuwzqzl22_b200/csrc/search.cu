@@ -15,9 +15,11 @@ cudaError_t launch_search(const SearchLaunch& a, cudaStream_t s) {
   if (a.nq == 0) return cudaSuccess;
   switch (nv4_for(a.d)) {
     case 1: return launch_search_nv<1>(a, s);
+#ifndef GANNS_DEV_NV1
     case 2: return launch_search_nv<2>(a, s);
     case 4: return launch_search_nv<4>(a, s);
     case 8: return launch_search_nv<8>(a, s);
+#endif
   }
   return cudaErrorInvalidValue;
 }

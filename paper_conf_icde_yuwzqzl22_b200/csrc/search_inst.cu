@@ -10,22 +10,28 @@
 
 namespace ganns {
 
+// Persistent: every warp pulls queries from a per-launch ticket counter until
+// the batch is exhausted, so the last wave is balanced at query granularity.
 template <int NV4, int TPL, bool L2>
-__global__ void __launch_bounds__(kWarpsPerBlock * 32)
+__global__ void __launch_bounds__(kSearchWarps * 32, kMinBlocksPerSM)
 search_kernel(GraphView g, const float* __restrict__ Q, int64_t nq, int k, int l, int e,
               int32_t entry, int32_t* __restrict__ out_ids, float* __restrict__ out_dists,
-              uint32_t* __restrict__ stats) {
+              uint32_t* __restrict__ stats, int32_t* __restrict__ ticket) {
   extern __shared__ __align__(16) uint8_t smem[];
   const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int64_t q = int64_t(blockIdx.x) * kWarpsPerBlock + w;
-  if (q >= nq) return;
-  uint8_t* base = smem + size_t(w) * warp_smem_bytes(l, TPL);
-  uint64_t* sN = reinterpret_cast<uint64_t*>(base);
-  uint64_t* sT = sN + lpad32(l);
-  uint32_t* sBM = reinterpret_cast<uint32_t*>(sT + TPL * 32);
+  WarpSmem ws = carve_warp_smem(smem + size_t(w) * warp_smem_bytes(l, TPL, NV4, g.d4), l, TPL,
+                                NV4, g.d4);
+  if (lane == 0) mbar_init(ws.mbar, 1);
+  __syncwarp();
+  uint64_t* sN = ws.sN;
+  for (;;) {
+  int32_t qt = 0;
+  if (lane == 0) qt = atomicAdd(ticket, 1);
+  const int64_t q = __shfl_sync(kFull, qt, 0);
+  if (q >= nq) break;
   SearchStats st;
   const int cnt = warp_search<NV4, TPL, L2, false>(g, Q + size_t(q) * (g.d4 * 4), entry, l, e,
-                                                   sN, sT, sBM, st);
+                                                   ws, st);
   // output: the first k of N, (-1, +inf) padded (R-C8)
   for (int i = lane; i < k; i += 32) {
     uint64_t key = i < cnt ? unflag(sN[i]) : kKeyInf;
@@ -38,33 +44,53 @@ search_kernel(GraphView g, const float* __restrict__ Q, int64_t nq, int k, int l
     stats[size_t(q) * 3 + 1] = st.comps;
     stats[size_t(q) * 3 + 2] = st.merged;
   }
+  __syncwarp();
+  }
 }
 
 template <int NV4, int TPL, bool L2>
 static cudaError_t launch_t(const SearchLaunch& a, cudaStream_t s) {
   auto kern = search_kernel<NV4, TPL, L2>;
-  const size_t smem = size_t(kWarpsPerBlock) * warp_smem_bytes(a.l, TPL);
+  const size_t smem = size_t(kSearchWarps) * warp_smem_bytes(a.l, TPL, NV4, a.d / 4);
   static bool attr_done = false;   // per instantiation
   if (!attr_done) {
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         int(kWarpsPerBlock * warp_smem_bytes(1024, TPL)));
+                                         227 * 1024);
+    if (e == cudaSuccess)
+      e = cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
     if (e != cudaSuccess) return e;
     attr_done = true;
   }
+  if (smem > 227 * 1024) return cudaErrorInvalidValue;
   GraphView g{a.nbr, a.X, a.n, a.d_max, a.d / 4, a.metric};
-  const int64_t blocks = (a.nq + kWarpsPerBlock - 1) / kWarpsPerBlock;
-  kern<<<dim3(unsigned(blocks)), kWarpsPerBlock * 32, smem, s>>>(
-      g, a.Q, a.nq, a.k, a.l, a.e, a.entry, a.out_ids, a.out_dists, a.stats);
+  int dev = 0, sms = 0, per_sm = 0;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  cudaError_t err = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kSearchWarps * 32, smem);
+  if (err != cudaSuccess) return err;
+  int64_t blocks = (a.nq + kSearchWarps - 1) / kSearchWarps;
+  const int64_t resident = int64_t(sms) * (per_sm > 0 ? per_sm : 1);
+  if (blocks > resident) blocks = resident;
+  err = cudaMemsetAsync(a.ticket, 0, sizeof(int32_t), s);
+  if (err != cudaSuccess) return err;
+  kern<<<dim3(unsigned(blocks)), kSearchWarps * 32, smem, s>>>(
+      g, a.Q, a.nq, a.k, a.l, a.e, a.entry, a.out_ids, a.out_dists, a.stats, a.ticket);
   count_launch();
   return cudaGetLastError();
 }
 
 template <int NV4, int TPL>
 static cudaError_t launch_m(const SearchLaunch& a, cudaStream_t s) {
+#ifdef GANNS_DEV_ONE
+  return launch_t<NV4, TPL, true>(a, s);
+#endif
   return a.metric == 0 ? launch_t<NV4, TPL, true>(a, s) : launch_t<NV4, TPL, false>(a, s);
 }
 template <int NV4>
 cudaError_t launch_search_nv(const SearchLaunch& a, cudaStream_t s) {
+#ifdef GANNS_DEV_ONE
+  return launch_m<NV4, 1>(a, s);
+#endif
   switch (tpl_for(a.d_max)) {
     case 1: return launch_m<NV4, 1>(a, s);
     case 2: return launch_m<NV4, 2>(a, s);
