@@ -1,0 +1,112 @@
+"""World-size-2 gloo tests of the multi-GPU orchestration (dist.py) on CPU.
+
+The per-rank search / merge are the oracle's (tests may call the oracle); what is
+under test is the host logic: query slicing, shard bounds, id offsets, the
+all-gather of per-shard [nq, k] lists and the merge order -- the same code that
+drives the sm_100a kernels over NCCL on B200s.
+"""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+import oracle
+import ganns_synth as syn
+from paper_conf_icde_yuwzqzl22_b200 import dist as gd
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _data():
+    cfg = syn.with_size(syn.CONFIGS["C1"], n=3000, nq=37)
+    return syn.points(cfg), syn.queries(cfg)
+
+
+def _worker(rank, world, port, out_dir):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    X, Q = _data()
+    k, l = 10, 48
+    # replicated graph, query data-parallel
+    nbr, _, _ = oracle.alg2(X, 8, 16, 256, l_build=32)
+
+    def search_full(q):
+        i, d = oracle.search(nbr, X, q.numpy(), k, l)
+        return torch.from_numpy(i), torch.from_numpy(d)
+
+    ri, rd = gd.search_replicated(search_full, torch.from_numpy(Q))
+    # sharded base set: each rank builds its own shard graph
+    lo, hi = gd.shard_bounds(len(X), rank, world)
+    snbr, _, _ = oracle.alg2(X[lo:hi], 8, 16, 128, l_build=32)
+
+    def search_shard(q):
+        i, d = oracle.search(snbr, X[lo:hi], q.numpy(), k, l)
+        return torch.from_numpy(i), torch.from_numpy(d)
+
+    def merge(i, d):
+        mi, md = oracle.merge_topk(i.numpy(), d.numpy())
+        return torch.from_numpy(mi), torch.from_numpy(md)
+
+    def offset(i, off):
+        return torch.where(i >= 0, i + off, i)
+
+    idx = gd.ShardedIndex(len(X), search_shard, merge, offset)
+    si, sd = idx.search(torch.from_numpy(Q))
+    t = gd.max_over_ranks(float(rank + 1))
+    np.savez(os.path.join(out_dir, f"r{rank}.npz"), ri=ri.numpy(), rd=rd.numpy(),
+             si=si.numpy(), sd=sd.numpy(), t=t)
+    dist.destroy_process_group()
+
+
+@pytest.fixture(scope="module")
+def results(tmp_path_factory):
+    out = str(tmp_path_factory.mktemp("dist"))
+    mp.spawn(_worker, args=(2, _free_port(), out), nprocs=2, join=True)
+    return [dict(np.load(os.path.join(out, f"r{r}.npz"))) for r in range(2)]
+
+
+def test_slices_cover_the_batch():
+    for nq in (0, 1, 7, 10_000):
+        for w in (1, 2, 3, 8):
+            sl = [gd.query_slice(nq, r, w) for r in range(w)]
+            assert sl[0][0] == 0 and sl[-1][1] == nq
+            assert all(a[1] == b[0] for a, b in zip(sl, sl[1:]))
+            assert max(b - a for a, b in sl) - min(b - a for a, b in sl) <= 1
+
+
+def test_replicated_equals_single_process(results):
+    X, Q = _data()
+    nbr, _, _ = oracle.alg2(X, 8, 16, 256, l_build=32)
+    ri, rd = oracle.search(nbr, X, Q, 10, 48)
+    for r in results:
+        assert (r["ri"] == ri).all() and (r["rd"] == rd).all()
+
+
+def test_sharded_equals_sequential_shards_and_merge(results):
+    X, Q = _data()
+    parts_i, parts_d = [], []
+    for rank in range(2):
+        lo, hi = gd.shard_bounds(len(X), rank, 2)
+        snbr, _, _ = oracle.alg2(X[lo:hi], 8, 16, 128, l_build=32)
+        i, d = oracle.search(snbr, X[lo:hi], Q, 10, 48)
+        parts_i.append(np.where(i >= 0, i + lo, -1))
+        parts_d.append(d)
+    mi, md = oracle.merge_topk(np.stack(parts_i), np.stack(parts_d))
+    for r in results:
+        assert (r["si"] == mi).all() and (r["sd"] == md).all()
+        assert float(r["t"]) == 2.0        # max over ranks
+    # sharding can only help recall at equal l (each shard keeps its own top-l)
+    gt, _ = oracle.bruteforce(X, Q, 10)
+    nbr, _, _ = oracle.alg2(X, 8, 16, 256, l_build=32)
+    single, _ = oracle.search(nbr, X, Q, 10, 48)
+    assert oracle.recall(mi, gt) >= oracle.recall(single, gt) - 0.02
