@@ -14,12 +14,12 @@ ap = argparse.ArgumentParser()
 ap.add_argument("--config", default="C2")
 ap.add_argument("--l", type=int, default=96)
 ap.add_argument("--reps", type=int, default=4)
-ap.add_argument("--graph-cache", default="/tmp/ganns_prof_graph.bin")
+ap.add_argument("--l-build", type=int, default=128)
 a = ap.parse_args()
 cfg = syn.CONFIGS[a.config]
 X = torch.from_numpy(syn.points(cfg)).cuda()
 Q = torch.from_numpy(syn.queries(cfg)).cuda()
-graph = g.build(X, metric=cfg.metric, degree=cfg.degree)
+graph = g.build(X, metric=cfg.metric, degree=cfg.degree, l_build=a.l_build)
 flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
 for _ in range(a.reps):
     flush.zero_()
