@@ -398,11 +398,16 @@ __device__ int warp_search(const GraphView& g, const float* __restrict__ qrow, i
   int hint = 0;   // every position < hint is explored
   const int lim_e = e < l ? e : l;
 
+  // speculation: the adjacency row of the second unexplored entry is loaded
+  // together with the first one's; if that vertex is the next one explored, its
+  // row is already in registers (saves one dependent global load per hit)
+  int32_t spec_v = -1;
+  int32_t spec_u[TPL];
   for (;;) {
-    // (1) candidate locating
+    // (1) candidate locating: first unexplored entry of N[0..min(e,|N|))
     const int lim = lim_e < cnt ? lim_e : cnt;
     int found = -1;
-    int32_t v = 0;
+    int32_t v = 0, w = -1;
     for (int c = hint >> 5; (c << 5) < lim; ++c) {
       int p = (c << 5) + lane;
       uint64_t k = p < lim ? sN[p] : kKeyInf;
@@ -412,6 +417,9 @@ __device__ int warp_search(const GraphView& g, const float* __restrict__ qrow, i
         found = (c << 5) + src;
         if (lane == src) sN[p] = k | kExplored;   // mark explored
         v = __shfl_sync(kFull, key_id(k), src);
+        const unsigned b2 = b & (b - 1);
+        const int32_t wk = __shfl_sync(kFull, key_id(k), b2 ? __ffs(b2) - 1 : 0);
+        w = b2 ? wk : -1;
         break;
       }
     }
@@ -419,12 +427,18 @@ __device__ int warp_search(const GraphView& g, const float* __restrict__ qrow, i
     st.iters++;
     // (2) neighbourhood exploration: T <- out-neighbours of v
     int32_t u[TPL];
+    const bool hit = v == spec_v;
     const int32_t* row = g.nbr + size_t(v) * g.d_max;
+    const int32_t* wrow = g.nbr + size_t(w < 0 ? 0 : w) * g.d_max;
 #pragma unroll
     for (int t = 0; t < TPL; ++t) {
-      int j = t * 32 + lane;
-      u[t] = j < g.d_max ? load_nbr<COHERENT>(row + j) : -1;
+      const int j = t * 32 + lane;
+      const int32_t ur = (!hit && j < g.d_max) ? load_nbr<COHERENT>(row + j) : -1;
+      const int32_t uw = (w >= 0 && j < g.d_max) ? load_nbr<COHERENT>(wrow + j) : -1;
+      u[t] = hit ? spec_u[t] : ur;
+      spec_u[t] = uw;
     }
+    spec_v = w;
     // (3) bulk distance computation
     if constexpr (!uses_tma(NV4)) {
 #pragma unroll
@@ -449,17 +463,22 @@ __device__ int warp_search(const GraphView& g, const float* __restrict__ qrow, i
 #pragma unroll
     for (int t = 0; t < TPL; ++t) {
       cand[t] = u[t] >= 0 && key[t] < worst;
-      rN[t] = 0;
-      if (cand[t]) {
-        int lo = 0, hi = cnt;   // lower_bound of key[t] in N[0..cnt)
-        while (lo < hi) {
-          int mid = (lo + hi) >> 1;
-          if (unflag(sN[mid]) < key[t]) lo = mid + 1;
-          else hi = mid;
-        }
-        rN[t] = lo;
-        if (lo < cnt && unflag(sN[lo]) == key[t]) cand[t] = false;
+      // 4-ary lower_bound of key[t] in N[0..cnt): three independent probes per
+      // step; the trip count depends only on cnt (warp-uniform)
+      const uint64_t kt = key[t];
+      int base = 0, len = cnt;   // invariant: lower_bound in [base, base + len]
+      while (len > 3) {
+        const int q = len >> 2;
+        const int c = (unflag(sN[base + q]) < kt ? 1 : 0) + (unflag(sN[base + 2 * q]) < kt ? 1 : 0) +
+                      (unflag(sN[base + 3 * q]) < kt ? 1 : 0);
+        base += c * q;
+        len = c < 3 ? q : len - 3 * q;
       }
+      int r = base;
+#pragma unroll
+      for (int i = 0; i < 3; ++i) r += (i < len && unflag(sN[base + i]) < kt) ? 1 : 0;
+      rN[t] = r;
+      if (r < cnt && unflag(sN[r]) == kt) cand[t] = false;   // lazy check: in N (R-C1)
       cb[t] = __ballot_sync(kFull, cand[t]);
       ncand += __popc(cb[t]);
     }
@@ -475,24 +494,35 @@ __device__ int warp_search(const GraphView& g, const float* __restrict__ qrow, i
 #pragma unroll
     for (int s = 0; s < TPL; ++s) {
       unsigned m = cb[s];
-      while (m) {
-        int src = __ffs(m) - 1;
-        m &= m - 1;
-        uint64_t ks = shfl64(key[s], src);
+      while (m) {   // four survivors per round: independent shuffles in flight
+        int src[4];
 #pragma unroll
-        for (int t = 0; t < TPL; ++t) rT[t] += (ks < key[t]) ? 1 : 0;
+        for (int i = 0; i < 4; ++i) {
+          src[i] = m ? __ffs(m) - 1 : -1;
+          m &= m ? m - 1 : 0u;
+        }
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+          const uint64_t ks = shfl64(key[s], src[i] < 0 ? 0 : src[i]);
+#pragma unroll
+          for (int t = 0; t < TPL; ++t) rT[t] += (src[i] >= 0 && ks < key[t]) ? 1 : 0;
+        }
       }
     }
     // (6) candidate update: merge T into N keeping l entries
-    int pmin = lp;
+    int pmin = lp, nins = 0;
 #pragma unroll
     for (int t = 0; t < TPL; ++t) {
-      int pos = rN[t] + rT[t];
-      if (cand[t] && pos < l) {
+      const int pos = rN[t] + rT[t];
+      const bool ins = cand[t] && pos < l;
+      if (ins) {
+        // a new candidate is likely to be explored soon: warm its adjacency row in L2
+        asm volatile("prefetch.global.L2 [%0];" ::"l"(g.nbr + size_t(u[t]) * g.d_max));
         sT[rT[t]] = key[t];
         atomicOr(&sBM[pos >> 5], 1u << (pos & 31));
         pmin = pos < pmin ? pos : pmin;
       }
+      nins += __popc(__ballot_sync(kFull, ins));
     }
 #pragma unroll
     for (int off = 16; off >= 1; off >>= 1) {
@@ -500,30 +530,25 @@ __device__ int warp_search(const GraphView& g, const float* __restrict__ qrow, i
       pmin = o < pmin ? o : pmin;
     }
     const int ncnt = cnt + ncand < l ? cnt + ncand : l;
-    if (pmin < l) {
+    if (nins > 0) {
       __syncwarp();
-      uint32_t bmw = lane < nwords ? sBM[lane] : 0u;
-      uint32_t pc = __popc(bmw), ex = pc;
-#pragma unroll
-      for (int off = 1; off < 32; off <<= 1) {
-        uint32_t o = __shfl_up_sync(kFull, ex, off);
-        if (lane >= off) ex += o;
-      }
-      ex -= pc;   // exclusive prefix of popcounts
-      st.merged += __shfl_sync(kFull, ex + pc, 31);
+      st.merged += nins;
+      // rebuild N in place from the last chunk down: output p takes the compacted
+      // T entry #(T positions < p) or N[p - #(T positions < p)]
+      int suffix = 0;   // T positions at or above the current chunk
       for (int c = (ncnt - 1) >> 5; c >= (pmin >> 5); --c) {
-        uint32_t word = __shfl_sync(kFull, bmw, c);
-        uint32_t base = __shfl_sync(kFull, ex, c);
-        int p = (c << 5) + lane;
-        bool isT = (word >> lane) & 1u;
-        int tb = int(base + __popc(word & lanemask_lt()));
+        const uint32_t word = sBM[c];
+        suffix += __popc(word);
+        const int p = (c << 5) + lane;
+        const bool isT = (word >> lane) & 1u;
+        const int tb = nins - suffix + __popc(word & lanemask_lt());
         uint64_t val = 0;
         if (p < ncnt) val = isT ? sT[tb] : sN[p - tb];
         __syncwarp();
         if (p < ncnt) sN[p] = val;
+        if (lane == 0) sBM[c] = 0u;
         __syncwarp();
       }
-      if (lane < nwords) sBM[lane] = 0u;
       hint = pmin < found + 1 ? pmin : found + 1;
     } else {
       hint = found + 1;
