@@ -39,7 +39,7 @@
 
 namespace ganns {
 
-constexpr int kBuildWarps = 4;
+constexpr int kBuildWarps = 1;   // one warp per CTA spreads the latency-bound build searches over all SMs
 
 // Insert key kx into a warp-distributed ascending row of d_max keys (TPL per
 // lane, slot j = t*32 + lane); the last key falls off when the row is full
@@ -121,8 +121,9 @@ phase1_kernel(BuildDev B, int64_t group_size, int64_t ngroups) {
   const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int64_t gi = int64_t(blockIdx.x) * kBuildWarps + w;
   if (gi >= ngroups) return;
-  WarpSmem ws = carve_warp_smem(smem + size_t(w) * warp_smem_bytes(B.l_build, TPL, NV4, B.g.d4),
-                                B.l_build, TPL, NV4, B.g.d4);
+  WarpSmem ws = carve_warp_smem(
+      smem + size_t(w) * warp_smem_bytes(B.l_build, TPL, NV4, B.g.d4, kBuildStageRounds),
+      B.l_build, TPL, NV4, B.g.d4, kBuildStageRounds);
   if (lane == 0) mbar_init(ws.mbar, 1);
   __syncwarp();
   uint64_t* sN = ws.sN;
@@ -168,8 +169,9 @@ round_search_kernel(BuildDev B, int64_t lo, int64_t hi, int32_t* __restrict__ Eu
   const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int64_t v = lo + int64_t(blockIdx.x) * kBuildWarps + w;
   if (v >= hi) return;
-  WarpSmem ws = carve_warp_smem(smem + size_t(w) * warp_smem_bytes(B.l_build, TPL, NV4, B.g.d4),
-                                B.l_build, TPL, NV4, B.g.d4);
+  WarpSmem ws = carve_warp_smem(
+      smem + size_t(w) * warp_smem_bytes(B.l_build, TPL, NV4, B.g.d4, kBuildStageRounds),
+      B.l_build, TPL, NV4, B.g.d4, kBuildStageRounds);
   if (lane == 0) mbar_init(ws.mbar, 1);
   __syncwarp();
   uint64_t* sN = ws.sN;
@@ -370,7 +372,8 @@ static int build_t(BuildArgs& a, cudaStream_t s) {
   B.l_build = a.l_build;
   B.e_build = a.e_build;
   B.stats = stats.p;
-  const size_t smem = size_t(kBuildWarps) * warp_smem_bytes(a.l_build, TPL, NV4, a.d / 4);
+  const size_t smem =
+      size_t(kBuildWarps) * warp_smem_bytes(a.l_build, TPL, NV4, a.d / 4, kBuildStageRounds);
   if (smem > 227 * 1024) return fail(-4, "build: shared memory per CTA exceeds 227 KB");
 
   // Phase 1 (lines 2-8): all local graphs in parallel, one warp per group

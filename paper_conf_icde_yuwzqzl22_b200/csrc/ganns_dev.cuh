@@ -140,16 +140,16 @@ struct SearchStats {
 // Per-warp shared memory: [stage: 32 vector rows, TMA destination][N][T][mbar][bitmap]
 __host__ __device__ constexpr int lpad32(int l) { return (l + 31) & ~31; }
 __host__ __device__ constexpr bool uses_tma(int nv4) { return nv4 <= 2; }
-#ifndef GANNS_STAGE_ROUNDS
-#define GANNS_STAGE_ROUNDS 2
-#endif
-constexpr int kStageRounds = GANNS_STAGE_ROUNDS;   // rows are staged in kStageRounds TMA rounds
-constexpr int kStageRows = 32 / kStageRounds;
-__host__ __device__ constexpr size_t stage_bytes(int nv4, int d4) {
-  return uses_tma(nv4) ? size_t(kStageRows) * d4 * 16 : 0;
+// The <= 32 rows of one exploration are staged in `rounds` TMA rounds (1 or 2):
+// 2 rounds halve the stage (more resident warps, the throughput-bound batched
+// search); 1 round saves a memory round trip (the latency-bound build).
+constexpr int kSearchStageRounds = 2;
+constexpr int kBuildStageRounds = 1;
+__host__ __device__ constexpr size_t stage_bytes(int nv4, int d4, int rounds) {
+  return uses_tma(nv4) ? size_t(32 / rounds) * d4 * 16 : 0;
 }
-__host__ __device__ constexpr size_t warp_smem_bytes(int l, int tpl, int nv4, int d4) {
-  return stage_bytes(nv4, d4) + size_t(lpad32(l)) * 8 + size_t(tpl) * 32 * 8 + 16 + 128;
+__host__ __device__ constexpr size_t warp_smem_bytes(int l, int tpl, int nv4, int d4, int rounds) {
+  return stage_bytes(nv4, d4, rounds) + size_t(lpad32(l)) * 8 + size_t(tpl) * 32 * 8 + 16 + 128;
 }
 struct WarpSmem {
   float4* stage;
@@ -158,11 +158,14 @@ struct WarpSmem {
   uint64_t* mbar;
   uint32_t* sBM;
   uint32_t phase;   // parity of the next mbarrier phase to wait for
+  int rounds;       // TMA rounds per exploration (1 or 2)
 };
-__device__ __forceinline__ WarpSmem carve_warp_smem(uint8_t* base, int l, int tpl, int nv4, int d4) {
+__device__ __forceinline__ WarpSmem carve_warp_smem(uint8_t* base, int l, int tpl, int nv4, int d4,
+                                                   int rounds) {
   WarpSmem w;
+  w.rounds = rounds;
   w.stage = reinterpret_cast<float4*>(base);
-  w.sN = reinterpret_cast<uint64_t*>(base + stage_bytes(nv4, d4));
+  w.sN = reinterpret_cast<uint64_t*>(base + stage_bytes(nv4, d4, rounds));
   w.sT = w.sN + lpad32(l);
   w.mbar = w.sT + tpl * 32;
   w.sBM = reinterpret_cast<uint32_t*>(w.mbar + 2);
@@ -220,13 +223,13 @@ __device__ __forceinline__ uint64_t accum4(uint64_t acc, const float4& q, const 
 // row j's total.
 // Gather: the rows of the passes of one round are fetched by TMA bulk copies
 // (one cp.async.bulk per lane that owns a row of the round) into the warp's
-// stage buffer and waited for with a single mbarrier phase -- kStageRounds
-// memory round trips per iteration, no registers held in flight.
-template <int S, int C, bool L2, bool FULL>
+// stage buffer and waited for with a single mbarrier phase -- ROUNDS memory
+// round trips per iteration, no registers held in flight.
+template <int S, int C, bool L2, bool FULL, int ROUNDS>
 __device__ __forceinline__ float tma_dot(const GraphView& g, const float4 (&qv)[C],
                                          int32_t u_mine, int lane, WarpSmem& ws) {
-  static_assert(S % kStageRounds == 0, "passes must split evenly into rounds");
-  constexpr int PPR = S / kStageRounds;             // passes per round
+  static_assert(S % ROUNDS == 0, "passes must split evenly into rounds");
+  constexpr int PPR = S / ROUNDS;                   // passes per round
   const int sl = lane & (S - 1), seg = lane / S;
   const uint32_t rowbytes = uint32_t(g.d4) * 16u;
   // lane j = g + S*s holds the row of pass g of segment s; it is staged in round
@@ -238,7 +241,7 @@ __device__ __forceinline__ float tma_dot(const GraphView& g, const float4 (&qv)[
   for (int f = 0; f < C; ++f) coff[f] = (FULL || sl + S * f < g.d4) ? sl + S * f : g.d4 - 1;
   float p[S];
 #pragma unroll
-  for (int r = 0; r < kStageRounds; ++r) {
+  for (int r = 0; r < ROUNDS; ++r) {
     const bool mine = u_mine >= 0 && my_round == r;
     const unsigned vm = __ballot_sync(kFull, mine);
     if (vm) {
@@ -338,8 +341,12 @@ __device__ __forceinline__ float group_distances(const GraphView& g,
   const bool full = g.d4 == S * C;
   float dot;
   if constexpr (S < 32) {
-    dot = full ? tma_dot<S, C, L2, true>(g, qv, u_mine, lane, ws)
-               : tma_dot<S, C, L2, false>(g, qv, u_mine, lane, ws);
+    if (ws.rounds == 1)
+      dot = full ? tma_dot<S, C, L2, true, 1>(g, qv, u_mine, lane, ws)
+                 : tma_dot<S, C, L2, false, 1>(g, qv, u_mine, lane, ws);
+    else
+      dot = full ? tma_dot<S, C, L2, true, 2>(g, qv, u_mine, lane, ws)
+                 : tma_dot<S, C, L2, false, 2>(g, qv, u_mine, lane, ws);
   } else {
     dot = full ? warp_dot<C, L2, true>(g, qv, u_mine, lane)
                : warp_dot<C, L2, false>(g, qv, u_mine, lane);

@@ -19,8 +19,9 @@ search_kernel(GraphView g, const float* __restrict__ Q, int64_t nq, int k, int l
               uint32_t* __restrict__ stats, int32_t* __restrict__ ticket) {
   extern __shared__ __align__(16) uint8_t smem[];
   const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  WarpSmem ws = carve_warp_smem(smem + size_t(w) * warp_smem_bytes(l, TPL, NV4, g.d4), l, TPL,
-                                NV4, g.d4);
+  WarpSmem ws = carve_warp_smem(
+      smem + size_t(w) * warp_smem_bytes(l, TPL, NV4, g.d4, kSearchStageRounds), l, TPL, NV4, g.d4,
+      kSearchStageRounds);
   if (lane == 0) mbar_init(ws.mbar, 1);
   __syncwarp();
   uint64_t* sN = ws.sN;
@@ -51,7 +52,8 @@ search_kernel(GraphView g, const float* __restrict__ Q, int64_t nq, int k, int l
 template <int NV4, int TPL, bool L2>
 static cudaError_t launch_t(const SearchLaunch& a, cudaStream_t s) {
   auto kern = search_kernel<NV4, TPL, L2>;
-  const size_t smem = size_t(kSearchWarps) * warp_smem_bytes(a.l, TPL, NV4, a.d / 4);
+  const size_t smem =
+      size_t(kSearchWarps) * warp_smem_bytes(a.l, TPL, NV4, a.d / 4, kSearchStageRounds);
   static bool attr_done = false;   // per instantiation
   if (!attr_done) {
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
