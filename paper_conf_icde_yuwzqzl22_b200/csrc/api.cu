@@ -27,6 +27,59 @@ int cuda_fail(cudaError_t e, const char* what) {
 }
 void count_launch(uint64_t n) { g_launches.fetch_add(n, std::memory_order_relaxed); }
 
+// cuTensorMapEncodeTiled through the runtime's driver entry point (no link-time
+// dependency on libcuda).  Maps are cached per (pointer, n, d).
+typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*,
+                                  const cuuint64_t*, const cuuint64_t*, const cuuint32_t*,
+                                  const cuuint32_t*, CUtensorMapInterleave, CUtensorMapSwizzle,
+                                  CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+struct TmapCacheEntry {
+  const float* X = nullptr;
+  int64_t n = 0;
+  int d = 0;
+  CUtensorMap map;
+};
+static std::mutex g_tmap_mu;
+static TmapCacheEntry g_tmap_cache[8];
+static int g_tmap_next = 0;
+
+cudaError_t zero_tmap(CUtensorMap* out) {
+  std::memset(out, 0, sizeof(*out));
+  return cudaSuccess;
+}
+
+cudaError_t encode_row_tmap(const float* X, int64_t n, int d, CUtensorMap* out) {
+  std::lock_guard<std::mutex> lock(g_tmap_mu);
+  for (auto& e : g_tmap_cache)
+    if (e.X == X && e.n == n && e.d == d) {
+      *out = e.map;
+      return cudaSuccess;
+    }
+  static EncodeTiledFn enc = nullptr;
+  if (!enc) {
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", reinterpret_cast<void**>(&enc),
+                                cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess || !enc)
+      return cudaErrorNotSupported;
+  }
+  const cuuint64_t dims[2] = {cuuint64_t(d), cuuint64_t(n)};
+  const cuuint64_t strides[1] = {cuuint64_t(d) * 4};
+  const cuuint32_t box[2] = {cuuint32_t(d), 1};
+  const cuuint32_t es[2] = {1, 1};
+  CUresult r = enc(out, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(X), dims, strides,
+                   box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                   CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return cudaErrorInvalidValue;
+  TmapCacheEntry& e = g_tmap_cache[g_tmap_next];
+  g_tmap_next = (g_tmap_next + 1) % 8;
+  e.X = X;
+  e.n = n;
+  e.d = d;
+  e.map = *out;
+  return cudaSuccess;
+}
+
 static bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
 
 static int check_graph(const ganns_graph* g) {
@@ -283,9 +336,10 @@ int ganns_search_host(const ganns_graph* g, const float* points, const float* qu
       return fail(GANNS_ECUDA, "cudaEventCreate failed");
     P.device = dev;
   }
-  // chunking: at least 2 chunks to overlap copies with the search, each large
-  // enough to fill the GPU (~8 queries per SM warp slot).
-  int64_t chunk = std::max<int64_t>(2048, (nq + 3) / 4);
+  // chunking: every search launch pays a drain tail of about one query latency,
+  // so chunks must be large (>= 64K queries) for the H2D/search/D2H overlap to
+  // win; smaller batches go in one chunk (copies are ~5% of the search time).
+  int64_t chunk = std::max<int64_t>(65536, (nq + 3) / 4);
   if (chunk > nq) chunk = nq;
   const size_t need_q = size_t(chunk) * g->d, need_r = size_t(chunk) * k;
   if (need_q > P.cap_q || need_r > P.cap_r) {

@@ -116,8 +116,10 @@ __device__ __forceinline__ void add_stats(unsigned long long* st, const SearchSt
 // Phase 1: local graph construction (Alg. 2 lines 2-8).
 template <int NV4, int TPL, bool L2>
 __global__ void __launch_bounds__(kBuildWarps * 32)
-phase1_kernel(BuildDev B, int64_t group_size, int64_t ngroups) {
-  extern __shared__ __align__(16) uint8_t smem[];
+phase1_kernel(BuildDev B, int64_t group_size, int64_t ngroups,
+              const __grid_constant__ CUtensorMap tmap) {
+  B.g.tmap = &tmap;
+  extern __shared__ __align__(128) uint8_t smem[];
   const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int64_t gi = int64_t(blockIdx.x) * kBuildWarps + w;
   if (gi >= ngroups) return;
@@ -164,8 +166,10 @@ template <int NV4, int TPL, bool L2>
 __global__ void __launch_bounds__(kBuildWarps * 32)
 round_search_kernel(BuildDev B, int64_t lo, int64_t hi, int32_t* __restrict__ Eu,
                     float* __restrict__ Ed, int32_t* __restrict__ indeg,
-                    int32_t* __restrict__ touched, int32_t* __restrict__ counters) {
-  extern __shared__ __align__(16) uint8_t smem[];
+                    int32_t* __restrict__ touched, int32_t* __restrict__ counters,
+                    const __grid_constant__ CUtensorMap tmap) {
+  B.g.tmap = &tmap;
+  extern __shared__ __align__(128) uint8_t smem[];
   const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int64_t v = lo + int64_t(blockIdx.x) * kBuildWarps + w;
   if (v >= hi) return;
@@ -363,7 +367,9 @@ static int build_t(BuildArgs& a, cudaStream_t s) {
   GANNS_TRY(cudaGetLastError());
 
   BuildDev B;
-  B.g = GraphView{a.out_nbr, a.X, n, dmax, a.d / 4, a.metric};
+  B.g = GraphView{a.out_nbr, a.X, nullptr, n, dmax, a.d / 4, a.metric};
+  CUtensorMap tmap;
+  GANNS_TRY(uses_tma(NV4) ? encode_row_tmap(a.X, n, a.d, &tmap) : zero_tmap(&tmap));
   B.gid = a.out_nbr;
   B.gdist = gdist.p;
   B.gpid = gpid.p;
@@ -378,7 +384,7 @@ static int build_t(BuildArgs& a, cudaStream_t s) {
 
   // Phase 1 (lines 2-8): all local graphs in parallel, one warp per group
   phase1_kernel<NV4, TPL, L2><<<unsigned((ngroups + kBuildWarps - 1) / kBuildWarps),
-                                kBuildWarps * 32, smem, s>>>(B, S, ngroups);
+                                kBuildWarps * 32, smem, s>>>(B, S, ngroups, tmap);
   count_launch();
   GANNS_TRY(cudaGetLastError());
 
@@ -391,7 +397,7 @@ static int build_t(BuildArgs& a, cudaStream_t s) {
     GANNS_TRY(cudaMemsetAsync(counters.p, 0, sizeof(int32_t) * 2, s));
     round_search_kernel<NV4, TPL, L2><<<unsigned((nv + kBuildWarps - 1) / kBuildWarps),
                                         kBuildWarps * 32, smem, s>>>(
-        B, lo, hi, Eu.p, Ed.p, indeg.p, touched.p, counters.p);
+        B, lo, hi, Eu.p, Ed.p, indeg.p, touched.p, counters.p, tmap);
     const unsigned gs = unsigned(std::min<int64_t>((nslots + 255) / 256, 148 * 4));
     alloc_segments_kernel<<<gs, 256, 0, s>>>(touched.p, indeg.p, segoff.p, counters.p);
     scatter_edges_kernel<<<gs, 256, 0, s>>>(Eu.p, Ed.p, nslots, dm, lo, segoff.p, fill.p, seg.p);

@@ -28,6 +28,7 @@
 //       the position bitmap, from the last chunk down to the first changed one
 //       (P:210-212).  Duplicates never reach the merge.
 #pragma once
+#include <cuda.h>   // CUtensorMap (type only; the map is encoded on the host)
 #include <cstdint>
 #include <cuda_runtime.h>
 
@@ -126,6 +127,8 @@ __device__ __forceinline__ int32_t load_nbr(const int32_t* p) {
 struct GraphView {
   const int32_t* nbr;   // [n][d_max] ids, -1 padded
   const float* X;       // [n][d]
+  const CUtensorMap* tmap;   // 2-D map of X (box = 1 row) for TMA tile::gather4; the
+                             // address of the launching kernel's __grid_constant__ param
   int64_t n;
   int d_max;
   int d4;               // d / 4
@@ -149,7 +152,9 @@ __host__ __device__ constexpr size_t stage_bytes(int nv4, int d4, int rounds) {
   return uses_tma(nv4) ? size_t(32 / rounds) * d4 * 16 : 0;
 }
 __host__ __device__ constexpr size_t warp_smem_bytes(int l, int tpl, int nv4, int d4, int rounds) {
-  return stage_bytes(nv4, d4, rounds) + size_t(lpad32(l)) * 8 + size_t(tpl) * 32 * 8 + 16 + 128;
+  // rounded to 128 B: the stage (first) must be 128-B aligned for tensor TMA
+  return (stage_bytes(nv4, d4, rounds) + size_t(lpad32(l)) * 8 + size_t(tpl) * 32 * 8 + 16 + 128 +
+          127) & ~size_t(127);
 }
 struct WarpSmem {
   float4* stage;
@@ -242,17 +247,37 @@ __device__ __forceinline__ float tma_dot(const GraphView& g, const float4 (&qv)[
   float p[S];
 #pragma unroll
   for (int r = 0; r < ROUNDS; ++r) {
-    const bool mine = u_mine >= 0 && my_round == r;
-    const unsigned vm = __ballot_sync(kFull, mine);
+    // tile::gather4 (d % 8 == 0, so every group of 4 rows starts 128-B aligned):
+    // lane 4m of this round fetches the rows of lanes 4m..4m+3 into 4 consecutive
+    // stage slots with ONE TMA instruction; absent neighbours get an out-of-range
+    // row coordinate (zero-filled, no memory traffic).  Otherwise one 1-D bulk
+    // copy per row.
+    const bool g4 = (g.d4 & 1) == 0;
+    const int32_t uo = u_mine >= 0 ? u_mine : 0x7fffffff;
+    const int32_t u1 = __shfl_down_sync(kFull, uo, 1);
+    const int32_t u2 = __shfl_down_sync(kFull, uo, 2);
+    const int32_t u3 = __shfl_down_sync(kFull, uo, 3);
+    const bool issuer = g4 ? ((lane & 3) == 0 && my_round == r && (uo & u1 & u2 & u3) != 0x7fffffff)
+                           : (u_mine >= 0 && my_round == r);
+    const unsigned vm = __ballot_sync(kFull, issuer);
     if (vm) {
       __syncwarp();
       fence_proxy_async_smem();   // earlier generic reads of the stage precede the async writes
-      if (lane == 0) mbar_arrive_expect_tx(ws.mbar, uint32_t(__popc(vm)) * rowbytes);
+      if (lane == 0)
+        mbar_arrive_expect_tx(ws.mbar, uint32_t(__popc(vm)) * (g4 ? 4u : 1u) * rowbytes);
       __syncwarp();
-      if (mine)
-        tma_row(reinterpret_cast<char*>(ws.stage) + size_t(my_slot) * rowbytes,
-                reinterpret_cast<const char*>(g.X) + uint64_t(uint32_t(u_mine)) * rowbytes,
-                rowbytes, ws.mbar);
+      char* dst = reinterpret_cast<char*>(ws.stage) + size_t(my_slot) * rowbytes;
+      if (issuer) {
+        if (g4)
+          asm volatile(
+              "cp.async.bulk.tensor.2d.shared::cta.global.tile::gather4.mbarrier::complete_tx::bytes"
+              " [%0], [%1, {%2, %3, %4, %5, %6}], [%7];" ::"r"(smem_u32(dst)),
+              "l"(g.tmap), "r"(0), "r"(uo), "r"(u1), "r"(u2), "r"(u3), "r"(smem_u32(ws.mbar))
+              : "memory");
+        else
+          tma_row(dst, reinterpret_cast<const char*>(g.X) + uint64_t(uint32_t(u_mine)) * rowbytes,
+                  rowbytes, ws.mbar);
+      }
       mbar_wait(ws.mbar, ws.phase);
       ws.phase ^= 1u;
     }

@@ -1,6 +1,7 @@
 // ganns_internal.h -- host-side declarations shared by the .cu translation units
 // of libganns.so (not part of the public ABI; see include/ganns.h).
 #pragma once
+#include <cuda.h>
 #include <cuda_runtime.h>
 #include <atomic>
 #include <cstdint>
@@ -29,6 +30,9 @@ void set_error(const std::string& msg);
 int fail(int status, const std::string& msg);
 int cuda_fail(cudaError_t e, const char* what);
 void count_launch(uint64_t n = 1);
+// TMA tensor map of the point rows (2-D {d, n}, box {d, 1}) for tile::gather4.
+cudaError_t encode_row_tmap(const float* X, int64_t n, int d, CUtensorMap* out);
+cudaError_t zero_tmap(CUtensorMap* out);
 
 // Template selectors.
 inline int nv4_for(int d) {

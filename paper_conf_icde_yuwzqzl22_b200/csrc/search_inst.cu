@@ -4,6 +4,8 @@
 #include "ganns_dev.cuh"
 #include "ganns_internal.h"
 
+#include <cstdlib>
+
 #ifndef GANNS_NV4
 #error "compile with -DGANNS_NV4=<1|2|4|8>"
 #endif
@@ -16,8 +18,10 @@ template <int NV4, int TPL, bool L2>
 __global__ void __launch_bounds__(kSearchWarps * 32, kMinBlocksPerSM)
 search_kernel(GraphView g, const float* __restrict__ Q, int64_t nq, int k, int l, int e,
               int32_t entry, int32_t* __restrict__ out_ids, float* __restrict__ out_dists,
-              uint32_t* __restrict__ stats, int32_t* __restrict__ ticket) {
-  extern __shared__ __align__(16) uint8_t smem[];
+              uint32_t* __restrict__ stats, int32_t* __restrict__ ticket,
+              const __grid_constant__ CUtensorMap tmap) {
+  g.tmap = &tmap;
+  extern __shared__ __align__(128) uint8_t smem[];
   const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
   WarpSmem ws = carve_warp_smem(
       smem + size_t(w) * warp_smem_bytes(l, TPL, NV4, g.d4, kSearchStageRounds), l, TPL, NV4, g.d4,
@@ -52,7 +56,7 @@ search_kernel(GraphView g, const float* __restrict__ Q, int64_t nq, int k, int l
 template <int NV4, int TPL, bool L2>
 static cudaError_t launch_t(const SearchLaunch& a, cudaStream_t s) {
   auto kern = search_kernel<NV4, TPL, L2>;
-  const size_t smem =
+  size_t smem =
       size_t(kSearchWarps) * warp_smem_bytes(a.l, TPL, NV4, a.d / 4, kSearchStageRounds);
   static bool attr_done = false;   // per instantiation
   if (!attr_done) {
@@ -64,11 +68,22 @@ static cudaError_t launch_t(const SearchLaunch& a, cudaStream_t s) {
     attr_done = true;
   }
   if (smem > 227 * 1024) return cudaErrorInvalidValue;
-  GraphView g{a.nbr, a.X, a.n, a.d_max, a.d / 4, a.metric};
+  {
+    // developer knob (occupancy experiments): extra shared memory per CTA
+    static const long pad = [] {
+      const char* e = std::getenv("GANNS_DEBUG_SEARCH_SMEM_PAD");
+      return e ? std::atol(e) : 0L;
+    }();
+    smem += size_t(pad);
+  }
+  GraphView g{a.nbr, a.X, nullptr, a.n, a.d_max, a.d / 4, a.metric};
+  CUtensorMap tmap;
+  cudaError_t err = uses_tma(NV4) ? encode_row_tmap(a.X, a.n, a.d, &tmap) : zero_tmap(&tmap);
+  if (err != cudaSuccess) return err;
   int dev = 0, sms = 0, per_sm = 0;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-  cudaError_t err = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kSearchWarps * 32, smem);
+  err = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kSearchWarps * 32, smem);
   if (err != cudaSuccess) return err;
   int64_t blocks = (a.nq + kSearchWarps - 1) / kSearchWarps;
   const int64_t resident = int64_t(sms) * (per_sm > 0 ? per_sm : 1);
@@ -76,7 +91,7 @@ static cudaError_t launch_t(const SearchLaunch& a, cudaStream_t s) {
   err = cudaMemsetAsync(a.ticket, 0, sizeof(int32_t), s);
   if (err != cudaSuccess) return err;
   kern<<<dim3(unsigned(blocks)), kSearchWarps * 32, smem, s>>>(
-      g, a.Q, a.nq, a.k, a.l, a.e, a.entry, a.out_ids, a.out_dists, a.stats, a.ticket);
+      g, a.Q, a.nq, a.k, a.l, a.e, a.entry, a.out_ids, a.out_dists, a.stats, a.ticket, tmap);
   count_launch();
   return cudaGetLastError();
 }

@@ -17,6 +17,7 @@ ap.add_argument("--ls", default="64,128,256")
 ap.add_argument("--l-build", type=int, default=0)
 ap.add_argument("--group", type=int, default=0)
 ap.add_argument("--reps", type=int, default=5)
+ap.add_argument("--nq-mult", default="1", help="comma list: time batches of m x nq queries")
 a = ap.parse_args()
 cfg = syn.CONFIGS[a.config]
 X = torch.from_numpy(syn.points(cfg)).cuda()
@@ -42,6 +43,21 @@ for l in [int(x) for x in a.ls.split(",")]:
         e1.synchronize()
         ts.append(e0.elapsed_time(e1) / 1e3)
     t = sorted(ts)[len(ts) // 2]
+    for m in [int(x) for x in a.nq_mult.split(",")]:
+        if m == 1:
+            continue
+        Qm = Q.repeat(m, 1)
+        tm = []
+        for _ in range(a.reps):
+            flush.zero_()
+            e0, e1 = torch.cuda.Event(True), torch.cuda.Event(True)
+            e0.record()
+            g.search(graph, X, Qm, cfg.k, l)
+            e1.record()
+            e1.synchronize()
+            tm.append(e0.elapsed_time(e1) / 1e3)
+        tmm = sorted(tm)[len(tm) // 2]
+        print(json.dumps({"l": l, "nq": len(Qm), "ms": round(tmm * 1e3, 3), "qps": round(len(Qm) / tmm)}))
     print(json.dumps({"l": l, "recall": round(recall_at(ids, gt), 4), "ms": round(t * 1e3, 3),
                       "qps": round(len(Q) / t), "alg_GBps": round(byts / t / 1e9, 1),
                       "iters": round(float(st[:, 0].float().mean()), 1),
