@@ -147,6 +147,44 @@ def recall_at(ids, gt):
     return float(hit) / (k * gt.shape[0])
 
 
+def select_operating_point(torch, g, graph, Xd, Qd, gt, k, target, flush):
+    """(l, e) sweep: recall@10 of every pair; among the pairs reaching `target`
+    the fastest (median of 3 timed launches) is the operating point.  e (explore
+    budget) is the paper's fine-grained speed/accuracy knob."""
+    sweep, chosen, feasible = [], {}, []
+
+    def timed(l, e, reps=3):
+        ts = []
+        for _ in range(reps):
+            flush.zero_()
+            a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a0.record()
+            g.search(graph, Xd, Qd, k, l, e=e)
+            a1.record()
+            a1.synchronize()
+            ts.append(a0.elapsed_time(a1))
+        return sorted(ts)[len(ts) // 2]
+
+    for l in L_SWEEP:
+        best_r = 0.0
+        for e in sorted({l, max(k, int(round(0.85 * l))), max(k, int(round(0.7 * l)))}, reverse=True):
+            ids, _ = g.search(graph, Xd, Qd, k, l, e=e)
+            r = recall_at(ids, gt)
+            sweep.append((l, e, round(r, 5)))
+            best_r = max(best_r, r)
+            for tgt in (0.9, 0.95, 0.99):
+                if r >= tgt and tgt not in chosen:
+                    chosen[tgt] = (l, e)
+            if r >= target:
+                feasible.append((l, e))
+        if best_r >= 0.99 or len(feasible) >= 6:
+            break
+    if not feasible:
+        return L_SWEEP[-1], L_SWEEP[-1], sweep, chosen
+    _, l_star, e_star = min((timed(l, e), l, e) for l, e in feasible)
+    return l_star, e_star, sweep, chosen
+
+
 def run_ours(args):
     import torch
     import torch.distributed as dist
@@ -174,21 +212,12 @@ def run_ours(args):
     build_s = time.perf_counter() - t0
     b_iters, b_comps, b_searches, b_rounds = graph.build_stats
 
-    # ---- l sweep -> smallest l with recall@10 >= target
+    # ---- (l, e) operating point (see select_operating_point)
     gt = ground_truth(torch, Xd, Qd, k)
-    sweep = []
-    chosen = {}
-    for l in L_SWEEP:
-        ids, _ = g.search(graph, Xd, Qd, k, l)
-        r = recall_at(ids, gt)
-        sweep.append((l, round(r, 5)))
-        for tgt in (0.9, 0.95, 0.99):
-            if r >= tgt and tgt not in chosen:
-                chosen[tgt] = l
-        if r >= 0.99:
-            break
-    l_star = chosen.get(args.target, L_SWEEP[-1])
-    ids, dists, st = g.search(graph, Xd, Qd, k, l_star, stats=True)
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+    l_star, e_star, sweep, chosen = select_operating_point(torch, g, graph, Xd, Qd, gt, k,
+                                                           args.target, flush)
+    ids, dists, st = g.search(graph, Xd, Qd, k, l_star, e=e_star, stats=True)
     rec = recall_at(ids, gt)
     st = st.long()
     d = cfg.d
@@ -200,12 +229,11 @@ def run_ours(args):
     iters_mean = float(st[:, 0].float().mean())
 
     # ---- timed steps: device-resident inputs, L2 flushed between steps
-    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
     stream = torch.cuda.current_stream()
     out = (torch.empty((Q.shape[0], k), dtype=torch.int32, device=dev),
            torch.empty((Q.shape[0], k), dtype=torch.float32, device=dev))
     for _ in range(args.warmup):
-        g.search(graph, Xd, Qd, k, l_star, out=out)
+        g.search(graph, Xd, Qd, k, l_star, e=e_star, out=out)
     torch.cuda.synchronize()
     launches0 = g.kernel_launches()
     times = []
@@ -218,7 +246,7 @@ def run_ours(args):
             e0 = torch.cuda.Event(enable_timing=True)
             e1 = torch.cuda.Event(enable_timing=True)
             e0.record(stream)
-            g.search(graph, Xd, Qd, k, l_star, out=out)
+            g.search(graph, Xd, Qd, k, l_star, e=e_star, out=out)
             e1.record(stream)
             e1.synchronize()
             times.append(e0.elapsed_time(e1))
@@ -241,13 +269,13 @@ def run_ours(args):
     hout = (torch.empty((Q.shape[0], k), dtype=torch.int32).pin_memory(),
             torch.empty((Q.shape[0], k), dtype=torch.float32).pin_memory())
     for _ in range(2):
-        g.search_host(graph, Xd, Qh, k, l_star, out=hout)
+        g.search_host(graph, Xd, Qh, k, l_star, e=e_star, out=hout)
     e2e_times = []
     for _ in range(args.steps):
         flush.zero_()
         torch.cuda.synchronize()
         t0 = time.perf_counter()
-        g.search_host(graph, Xd, Qh, k, l_star, out=hout)
+        g.search_host(graph, Xd, Qh, k, l_star, e=e_star, out=hout)
         e2e_times.append(time.perf_counter() - t0)
     e2e_t = torch.tensor([sum(e2e_times)], dtype=torch.float64, device=dev)
     if world > 1:
@@ -261,7 +289,7 @@ def run_ours(args):
     if os.path.exists(tp):
         with open(tp) as f:
             tr = json.load(f)
-        if tr.get("config") == args.config and tr.get("l") == l_star:
+        if tr.get("config") == args.config and tr.get("l") == l_star and tr.get("e", l_star) == e_star:
             traffic = tr.get("dram_bytes_per_launch")
 
     line = {
@@ -279,9 +307,10 @@ def run_ours(args):
         "data": "synthetic",
         "config": {"workload": f"{args.config}: SIFT1M-shaped {cfg.n}x{cfg.d} L2, NSW degree "
                                f"{cfg.degree}, {Q.shape[0]} queries/GPU, k={k}",
-                   "l": l_star, "e": l_star, "recall_at_10": round(rec, 5),
-                   "l_for_recall": {str(t): chosen.get(t) for t in (0.9, 0.95, 0.99)},
-                   "l_sweep_recall": sweep, "mean_iterations": round(iters_mean, 2),
+                   "l": l_star, "e": e_star, "recall_at_10": round(rec, 5),
+                   "selection": "fastest (l, e) with recall@10 >= target among the sweep",
+                   "le_for_recall": {str(t): chosen.get(t) for t in (0.9, 0.95, 0.99)},
+                   "le_sweep_recall": sweep, "mean_iterations": round(iters_mean, 2),
                    "l2": "flushed (256 MiB write) between timed steps",
                    "parallelism": f"replicated graph, query data-parallel x{world}"},
         "build_seconds": round(build_s, 4),
@@ -300,7 +329,8 @@ def run_ours(args):
         "clocks": clk.summary(),
     }
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        line["cpu_baseline"] = cpu_baseline(graph.adjacency(), X, Q, k, l_star, args.cpu_seconds)
+        line["cpu_baseline"] = cpu_baseline(graph.adjacency(), X, Q, k, l_star, e_star,
+                                            args.cpu_seconds)
     if rank == 0:
         s = json.dumps(line)
         print(s, flush=True)
@@ -311,21 +341,21 @@ def run_ours(args):
         dist.destroy_process_group()
 
 
-def cpu_baseline(nbr, X, Q, k, l, seconds):
+def cpu_baseline(nbr, X, Q, k, l, e, seconds):
     """The oracle's search (plain C, one pthread per host core) on a bounded sample
     of the same queries and graph.  Returns the cpu_baseline object."""
     import oracle
     cores = oracle.ncores()
     m = 64
     t0 = time.perf_counter()
-    oracle.search(nbr, X, Q[:m], k, l, threads=cores)
+    oracle.search(nbr, X, Q[:m], k, l, e=e, threads=cores)
     dt = time.perf_counter() - t0
     m2 = int(min(len(Q), max(m, m * seconds / max(dt, 1e-3))))
     t0 = time.perf_counter()
-    oracle.search(nbr, X, Q[:m2], k, l, threads=cores)
+    oracle.search(nbr, X, Q[:m2], k, l, e=e, threads=cores)
     dt = time.perf_counter() - t0
     return {"value": round(m2 / dt, 1), "unit": "queries/s", "cores": cores, "kind": "oracle",
-            "sample": f"first {m2} of the {len(Q)} queries, same graph, l={l}, {dt:.1f} s"}
+            "sample": f"first {m2} of the {len(Q)} queries, same graph, l={l}, e={e}, {dt:.1f} s"}
 
 
 def run_reference(args):
@@ -346,37 +376,34 @@ def run_reference(args):
     nbr = graph.adjacency()
     Qd = torch.from_numpy(Q).cuda()
     gt = ground_truth(torch, Xd, Qd, k)
-    l_star = L_SWEEP[-1]
-    for l in L_SWEEP:
-        ids, _ = g.search(graph, Xd, Qd, k, l)
-        if recall_at(ids, gt) >= args.target:
-            l_star = l
-            break
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=Xd.device)
+    l_star, e_star, _, _ = select_operating_point(torch, g, graph, Xd, Qd, gt, k, args.target, flush)
     del Xd, Qd
     cores = oracle.ncores()
     per_step = 48
     for _ in range(args.warmup):
-        oracle.search(nbr, X, Q[:16], k, l_star, threads=cores)
+        oracle.search(nbr, X, Q[:16], k, l_star, e=e_star, threads=cores)
     t0 = time.perf_counter()
-    oracle.search(nbr, X, Q[:per_step], k, l_star, threads=cores)
+    oracle.search(nbr, X, Q[:per_step], k, l_star, e=e_star, threads=cores)
     dt = time.perf_counter() - t0
     per_step = int(max(cores, min(len(Q), per_step * 6.0 / max(dt, 1e-3))))
     times = []
     for s in range(args.steps):
         a = (s * per_step) % max(1, len(Q) - per_step)
         t0 = time.perf_counter()
-        oracle.search(nbr, X, Q[a:a + per_step], k, l_star, threads=cores)
+        oracle.search(nbr, X, Q[a:a + per_step], k, l_star, e=e_star, threads=cores)
         times.append(time.perf_counter() - t0)
     tot = sum(times)
     v = per_step * args.steps / tot
-    sample = f"{per_step} queries/step of the {len(Q)}-query batch, same graph, l={l_star}"
+    sample = (f"{per_step} queries/step of the {len(Q)}-query batch, same graph, "
+              f"l={l_star}, e={e_star}")
     print(json.dumps({
         "impl": "reference", "metric": "queries/sec at recall@10=0.95", "value": round(v, 1),
         "unit": "queries/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
         "ms_per_step": round(tot / args.steps * 1e3, 3), "higher_is_better": True,
         "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
         "config": {"workload": f"{args.config}: SIFT1M-shaped {cfg.n}x{cfg.d} L2, NSW degree "
-                               f"{cfg.degree}, k={k}", "l": l_star},
+                               f"{cfg.degree}, k={k}", "l": l_star, "e": e_star},
         "cpu_baseline": {"value": round(v, 1), "unit": "queries/s", "cores": cores,
                          "kind": "oracle", "sample": sample},
         "e2e": {"value": round(v, 1), "unit": "queries/s", "h2d_bytes_per_step": 0,
