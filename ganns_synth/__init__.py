@@ -150,3 +150,14 @@ def random_int_points(n: int, d: int, lo: int, hi: int, seed: int) -> np.ndarray
     """Small tie-heavy integer-grid point sets for oracle pins and edge cases."""
     rng = np.random.Generator(np.random.PCG64(np.random.SeedSequence([2022, 8, seed])))
     return rng.integers(lo, hi + 1, size=(n, d)).astype(np.float32)
+
+
+def hnsw_levels(n: int, d_min: int, seed: int) -> np.ndarray:
+    """Top layer of every point for the HNSW extension ("a subset ... randomly
+    selected", the higher the fewer): level = floor(-ln(U) * mL), U ~ U(0, 1],
+    mL = 1 / ln(d_min) (the standard HNSW normalisation, so each layer keeps about
+    1/d_min of the one below).  A seeded input, identical for the oracle and the GPU."""
+    rng = np.random.Generator(np.random.PCG64(np.random.SeedSequence([2022, 9, seed])))
+    u = 1.0 - rng.random(n)                      # (0, 1]
+    lv = np.floor(-np.log(u) / np.log(d_min)).astype(np.int64)
+    return np.minimum(lv, 15).astype(np.int8)

@@ -53,7 +53,11 @@ def lib():
         _lib.ora_alg2.argtypes = [P, i64, i32, i32, i32, i32, i32, i32, i64, i32, i32, P, P, P]
         _lib.ora_naive_parallel.argtypes = [P, i64, i32, i32, i32, i32, i32, i32, i64, P, P]
         _lib.ora_merge_topk.argtypes = [P, P, i32, i64, i32, P, P]
-        for f in ("ora_merge_topk", "ora_search_one", "ora_search_batch", "ora_alg1", "ora_bruteforce",
+        _lib.ora_hnsw_build.argtypes = [P, i64, i32, i32, P, i32, i32, i32, i32, i64, P, P, P,
+                                        P, P]
+        _lib.ora_hnsw_search.argtypes = [P, P, i32, P, P, i64, i32, P, i32, i32, P, i64, i32,
+                                         i32, i32, P, P, P, P]
+        for f in ("ora_hnsw_build", "ora_hnsw_search", "ora_merge_topk", "ora_search_one", "ora_search_batch", "ora_alg1", "ora_bruteforce",
                   "ora_nsw_seq", "ora_alg2", "ora_naive_parallel"):
             getattr(_lib, f).restype = ct.c_int
     return _lib
@@ -202,3 +206,44 @@ def merge_topk(ids, dists):
     od = np.empty((nq, k), np.float32)
     _check(lib().ora_merge_topk(_p(ids), _p(dists), W, nq, k, _p(oi), _p(od)))
     return oi, od
+
+
+def hnsw_build(X, levels, d_min, d_max, group_size, l_build=64, e_build=0, metric="l2"):
+    """HNSW (Section IV-D).  Returns dict(perm, layer_n, upper, layer0):
+    perm[new] = old; layer_n[j] = |layer j|; upper[j] (j >= 1) = [n_j, d_max] adjacency
+    in shuffled ids; layer0 = [n, d_max] adjacency in original ids."""
+    X = _f32(X)
+    levels = np.ascontiguousarray(levels, dtype=np.int8)
+    n = X.shape[0]
+    L = int(levels.max()) + 1
+    perm = np.empty(n, np.int32)
+    layer_n = np.zeros(L, np.int64)
+    nl = ct.c_int()
+    cnt = [int((levels >= j).sum()) for j in range(L)]
+    upper = np.empty(max(1, sum(cnt[1:]) * d_max), np.int32)
+    layer0 = np.empty((n, d_max), np.int32)
+    _check(lib().ora_hnsw_build(_p(X), n, X.shape[1], METRICS[metric], _p(levels), d_min, d_max,
+                                l_build, e_build, group_size, _p(perm), _p(layer_n),
+                                ct.byref(nl), _p(upper), _p(layer0)))
+    ups, off = {}, 0
+    for j in range(1, nl.value):
+        ups[j] = upper[off:off + cnt[j] * d_max].reshape(cnt[j], d_max).copy()
+        off += cnt[j] * d_max
+    return dict(perm=perm, layer_n=layer_n, upper=ups, layer0=layer0, upper_flat=upper)
+
+
+def hnsw_search(h, X, Q, k, l, e=0, metric="l2", stats=False):
+    """Greedy descent through the upper layers, then GANNS on layer 0.
+    Returns ids, dists, entries (+ stats [nq,4])."""
+    X, Q = _f32(X), _f32(np.atleast_2d(Q))
+    nq = Q.shape[0]
+    ids = np.empty((nq, k), np.int32)
+    dists = np.empty((nq, k), np.float32)
+    ent = np.empty(nq, np.int32)
+    st = np.empty((nq, 4), np.uint32) if stats else None
+    layer0 = h["layer0"]
+    _check(lib().ora_hnsw_search(_p(h["perm"]), _p(h["layer_n"]), len(h["layer_n"]),
+                                 _p(h["upper_flat"]), _p(layer0), layer0.shape[0],
+                                 layer0.shape[1], _p(X), X.shape[1], METRICS[metric], _p(Q), nq,
+                                 k, l, e, _p(ids), _p(dists), _p(st), _p(ent)))
+    return (ids, dists, ent, st) if stats else (ids, dists, ent)

@@ -311,3 +311,61 @@ def test_merge_topk_of_exact_shards_is_global_bruteforce(W):
     mi, md = oracle.merge_topk(np.stack(sid), np.stack(sd))
     gi, gd = oracle.bruteforce(X, Q, k, threads=1)
     assert (mi == gi).all() and (md == gd).all()
+
+
+# ------------------------------------------------ HNSW, NEXT-1
+def test_hnsw_levels_are_geometric():
+    lv = syn.hnsw_levels(200_000, 16, 1)
+    for j in (1, 2, 3):
+        frac = (lv >= j).mean()
+        assert abs(frac - 16.0 ** -j) < 4 * np.sqrt(16.0 ** -j / 200_000) + 1e-4
+
+
+def test_hnsw_layers_are_id_prefixes_and_exact_regime_is_sequential_nsw():
+    """With exact searches (l_build >= n, d_max >= n-1) every layer equals the
+    sequential NSW of its points taken in shuffled order (quality theorem per
+    layer), upper layers only reference ids of their prefix, and layer 0 is
+    that graph relabelled to the original ids (P:373 steps 1-3)."""
+    for seed in range(6):
+        n = 40 + seed * 3
+        X = syn.random_int_points(n, 4, 0, 6, 40 + seed)
+        levels = np.zeros(n, np.int8)
+        rng = np.random.default_rng(seed)
+        levels[rng.choice(n, 12, replace=False)] = 1
+        levels[rng.choice(np.nonzero(levels)[0], 4, replace=False)] = 2
+        h = oracle.hnsw_build(X, levels, 3, 64, group_size=7, l_build=n + 1)
+        perm, ln = h["perm"], h["layer_n"]
+        # perm: stable by level descending
+        order = sorted(range(n), key=lambda v: (-levels[v], v))
+        assert perm.tolist() == order
+        assert ln.tolist() == [n, 12, 4]
+        Xp = X[perm]
+        for j in (1, 2):
+            up = h["upper"][j]
+            assert up.max() < ln[j]
+            ref, _, _ = oracle.nsw_seq(Xp[:ln[j]], 3, 64, exact=True)
+            assert (up == ref).all()
+        ref0, _, _ = oracle.nsw_seq(Xp, 3, 64, exact=True)
+        relab = np.full_like(ref0, -1)
+        for v in range(n):
+            row = ref0[v]
+            relab[perm[v]] = np.where(row >= 0, perm[np.maximum(row, 0)], -1)
+        assert (h["layer0"] == relab).all()
+        # search: exact layer 0 search whatever the entry; the descent entry is the
+        # nearest top-layer point (greedy on complete upper layers)
+        Q = syn.random_int_points(5, 4, 0, 6, 90 + seed)
+        ids, dists, ent = oracle.hnsw_search(h, X, Q, 5, n + 1)
+        gi, gd = oracle.bruteforce(X, Q, 5)
+        assert (ids == gi).all() and (dists == gd).all()
+
+
+def test_hnsw_quality_at_least_nsw():
+    cfg = syn.with_size(syn.CONFIGS["C1"], n=4000, nq=100)
+    X, Q = syn.points(cfg), syn.queries(cfg)
+    gt, _ = oracle.bruteforce(X, Q, 10)
+    lv = syn.hnsw_levels(len(X), 8, 3)
+    h = oracle.hnsw_build(X, lv, 8, 16, group_size=128, l_build=32)
+    nsw, _, _ = oracle.alg2(X, 8, 16, 128, l_build=32)
+    ih, _, _ = oracle.hnsw_search(h, X, Q, 10, 32)
+    inn, _ = oracle.search(nsw, X, Q, 10, 32)
+    assert oracle.recall(ih, gt) >= oracle.recall(inn, gt) - 0.02

@@ -13,6 +13,7 @@ import paper_conf_icde_yuwzqzl22_b200 as g  # noqa: E402
 ap = argparse.ArgumentParser()
 ap.add_argument("--config", default="C2")
 ap.add_argument("--l", type=int, default=96)
+ap.add_argument("--e", type=int, default=0)
 ap.add_argument("--reps", type=int, default=4)
 ap.add_argument("--l-build", type=int, default=128)
 a = ap.parse_args()
@@ -23,6 +24,6 @@ graph = g.build(X, metric=cfg.metric, degree=cfg.degree, l_build=a.l_build)
 flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
 for _ in range(a.reps):
     flush.zero_()
-    g.search(graph, X, Q, cfg.k, a.l)
+    g.search(graph, X, Q, cfg.k, a.l, e=a.e)
 torch.cuda.synchronize()
 print("done", graph.build_stats)
