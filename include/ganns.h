@@ -162,6 +162,49 @@ GANNS_API int ganns_graph_load(const char *path, int device, ganns_graph **out);
 /* ganns_graph_free -- NULL is a no-op. */
 GANNS_API void ganns_graph_free(ganns_graph *g);
 
+/* ---------------------------------------------------------------- HNSW
+ * HNSW extension of Algorithm 2 (Section IV-D).  Layer j holds the
+ * points whose level >= j (levels are drawn by the caller -- the random
+ * selection of P:369 -- and passed in).  (1) ids are shuffled: points sorted by
+ * level descending, ties by id (perm[new] = old), so layer j is the shuffled-id
+ * prefix [0, n_j); (2) layers are built top-down with Algorithm 2 on their
+ * prefix; a Phase-2 search enters layer j at the vertex reached by a greedy
+ * descent (GANNS search with l = e = 1) of the finished layers above, if that
+ * vertex is already merged, else at vertex 0; (3) layer 0 is relabelled to the
+ * original ids (a plain ganns_graph); the upper layers stay in shuffled ids.
+ * Search = greedy descent of the upper layers, then the GANNS search on layer 0
+ * from the vertex reached. */
+typedef struct ganns_hnsw ganns_hnsw;
+
+/* ganns_build_hnsw -- as ganns_build, plus
+ *   levels_host  host int8 [n], level of every point, 0 <= level < 16.
+ * Syncs.  The index keeps a device copy of the rows of the upper-layer points. */
+GANNS_API int ganns_build_hnsw(const float *points, int64_t n, int d, int metric, int degree,
+                               const int8_t *levels_host, const ganns_build_params *p,
+                               void *stream, ganns_hnsw **out);
+
+/* ganns_hnsw_search -- ganns_search_ex on the HNSW index; p->entry is ignored
+ * (each query enters layer 0 where its descent ends).  Launches two kernels. */
+GANNS_API int ganns_hnsw_search(const ganns_hnsw *h, const float *points, const float *queries,
+                                int64_t nq, int k, int l, const ganns_search_params *p,
+                                int32_t *out_ids, float *out_dists, void *stream);
+
+/* ganns_hnsw_info -- number of layers; layer_n (nullable) receives n_j for j < nlayers. */
+GANNS_API int ganns_hnsw_info(const ganns_hnsw *h, int *nlayers, int64_t *layer_n);
+
+/* ganns_hnsw_layer -- copy layer j's adjacency to host out [n_j][d_max]: layer 0
+ * in original ids, layers >= 1 in shuffled ids.  Syncs. */
+GANNS_API int ganns_hnsw_layer(const ganns_hnsw *h, int layer, int32_t *out_host);
+
+/* ganns_hnsw_perm -- copy perm[n] (shuffled id -> original id) to host.  Syncs. */
+GANNS_API int ganns_hnsw_perm(const ganns_hnsw *h, int32_t *out_host);
+
+/* ganns_hnsw_base -- layer 0 as a ganns_graph (borrowed; valid until ganns_hnsw_free). */
+GANNS_API int ganns_hnsw_base(const ganns_hnsw *h, const ganns_graph **base);
+
+/* ganns_hnsw_free -- NULL is a no-op. */
+GANNS_API void ganns_hnsw_free(ganns_hnsw *h);
+
 /* ganns_last_error -- thread-local message of the last failing call ("" if none). */
 GANNS_API const char *ganns_last_error(void);
 

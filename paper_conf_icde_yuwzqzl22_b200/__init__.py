@@ -55,6 +55,12 @@ def _load():
         "ganns_graph_info": [P, ct.POINTER(i64), ct.POINTER(i32), ct.POINTER(i32), ct.POINTER(i32)],
         "ganns_graph_save": [P, ct.c_char_p],
         "ganns_graph_load": [ct.c_char_p, i32, ct.POINTER(P)],
+        "ganns_build_hnsw": [P, i64, i32, i32, i32, P, ct.POINTER(_BuildParams), P, ct.POINTER(P)],
+        "ganns_hnsw_search": [P, P, P, i64, i32, i32, ct.POINTER(_SearchParams), P, P, P],
+        "ganns_hnsw_info": [P, ct.POINTER(i32), P],
+        "ganns_hnsw_layer": [P, i32, P],
+        "ganns_hnsw_perm": [P, P],
+        "ganns_hnsw_base": [P, ct.POINTER(P)],
     }
     for name, args in sig.items():
         f = getattr(lib, name)
@@ -62,6 +68,8 @@ def _load():
         f.restype = ct.c_int
     lib.ganns_graph_free.argtypes = [P]
     lib.ganns_graph_free.restype = None
+    lib.ganns_hnsw_free.argtypes = [P]
+    lib.ganns_hnsw_free.restype = None
     lib.ganns_last_error.argtypes = []
     lib.ganns_last_error.restype = ct.c_char_p
     lib.ganns_kernel_launches.argtypes = []
@@ -76,7 +84,9 @@ ABI_SYMBOLS = ("ganns_build", "ganns_search", "ganns_search_ex", "ganns_search_h
                "ganns_merge_topk", "ganns_offset_ids", "ganns_graph_from_adjacency",
                "ganns_graph_adjacency", "ganns_graph_device_ptr", "ganns_graph_info",
                "ganns_graph_save", "ganns_graph_load", "ganns_graph_free", "ganns_last_error",
-               "ganns_kernel_launches")
+               "ganns_kernel_launches", "ganns_build_hnsw", "ganns_hnsw_search",
+               "ganns_hnsw_info", "ganns_hnsw_layer", "ganns_hnsw_perm", "ganns_hnsw_base",
+               "ganns_hnsw_free")
 
 
 def lib():
@@ -109,8 +119,9 @@ def kernel_launches() -> int:
 class Graph:
     """Fixed-degree proximity graph (int32 [n][d_max] adjacency in device memory)."""
 
-    def __init__(self, handle: ct.c_void_p):
+    def __init__(self, handle: ct.c_void_p, owned: bool = True):
         self._h = handle
+        self._owned = owned
         n, d, dm, m = ct.c_int64(), ct.c_int(), ct.c_int(), ct.c_int()
         _check(_lib.ganns_graph_info(handle, ct.byref(n), ct.byref(d), ct.byref(dm), ct.byref(m)))
         self.n, self.d, self.d_max, self.metric = n.value, d.value, dm.value, _METRIC_NAMES[m.value]
@@ -140,9 +151,9 @@ class Graph:
         return Graph(h)
 
     def free(self):
-        if self._h:
+        if self._h and self._owned:
             _lib.ganns_graph_free(self._h)
-            self._h = None
+        self._h = None
 
     def __del__(self):
         try:
@@ -243,3 +254,86 @@ def offset_ids(ids: torch.Tensor, offset: int, stream=None) -> torch.Tensor:
         _check(_lib.ganns_offset_ids(ct.c_void_p(ids.data_ptr()), ids.numel(), offset,
                                      _stream(stream)))
     return ids
+
+
+class Hnsw:
+    """HNSW index (Section IV-D): upper layers in shuffled ids + layer 0."""
+
+    def __init__(self, handle: ct.c_void_p):
+        self._h = handle
+        nl = ct.c_int()
+        ln = (ct.c_int64 * 16)()
+        _check(_lib.ganns_hnsw_info(handle, ct.byref(nl), ct.cast(ln, ct.c_void_p)))
+        self.nlayers = nl.value
+        self.layer_n = [int(ln[j]) for j in range(nl.value)]
+        b = ct.c_void_p()
+        _check(_lib.ganns_hnsw_base(handle, ct.byref(b)))
+        self.base = Graph(b, owned=False)
+        self.build_stats = None
+
+    @property
+    def handle(self):
+        return self._h
+
+    def layer(self, j: int) -> np.ndarray:
+        out = np.empty((self.layer_n[j], self.base.d_max), np.int32)
+        _check(_lib.ganns_hnsw_layer(self._h, j, out.ctypes.data_as(ct.c_void_p)))
+        return out
+
+    def perm(self) -> np.ndarray:
+        out = np.empty(self.layer_n[0], np.int32)
+        _check(_lib.ganns_hnsw_perm(self._h, out.ctypes.data_as(ct.c_void_p)))
+        return out
+
+    def free(self):
+        if self._h:
+            self.base._h = None
+            _lib.ganns_hnsw_free(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.free()
+        except Exception:
+            pass
+
+
+def build_hnsw(points: torch.Tensor, levels: np.ndarray, metric: str = "l2", degree: int = 32,
+               d_min: int = 0, l_build: int = 0, e_build: int = 0, group_size: int = 0,
+               stream=None) -> Hnsw:
+    """HNSW construction: Algorithm 2 per layer, top-down.  `levels`
+    int8 [n] (e.g. ganns_synth.hnsw_levels)."""
+    points = _dev_f32(points, "points")
+    levels = np.ascontiguousarray(levels, dtype=np.int8)
+    st = (ct.c_uint64 * 4)()
+    p = _BuildParams(d_min, l_build, e_build, group_size, 0, 0, ct.cast(st, ct.POINTER(ct.c_uint64)))
+    h = ct.c_void_p()
+    with torch.cuda.device(points.device):
+        _check(_lib.ganns_build_hnsw(ct.c_void_p(points.data_ptr()), points.shape[0],
+                                     points.shape[1], METRICS[metric], degree,
+                                     levels.ctypes.data_as(ct.c_void_p), ct.byref(p),
+                                     _stream(stream), ct.byref(h)))
+    idx = Hnsw(h)
+    idx.build_stats = tuple(int(x) for x in st)
+    return idx
+
+
+def hnsw_search(index: Hnsw, points: torch.Tensor, queries: torch.Tensor, k: int, l: int,
+                e: int = 0, stats: bool = False, out=None, stream=None):
+    """Greedy descent of the upper layers, then the GANNS search on layer 0."""
+    points = _dev_f32(points, "points")
+    queries = _dev_f32(queries, "queries")
+    nq = queries.shape[0]
+    if out is None:
+        ids = torch.empty((nq, k), dtype=torch.int32, device=queries.device)
+        dists = torch.empty((nq, k), dtype=torch.float32, device=queries.device)
+    else:
+        ids, dists = out
+    st = torch.empty((nq, 3), dtype=torch.int32, device=queries.device) if stats else None
+    p = _SearchParams(e, 0, ct.c_void_p(st.data_ptr()) if stats else None)
+    with torch.cuda.device(queries.device):
+        _check(_lib.ganns_hnsw_search(index.handle, ct.c_void_p(points.data_ptr()),
+                                      ct.c_void_p(queries.data_ptr()), nq, k, l, ct.byref(p),
+                                      ct.c_void_p(ids.data_ptr()), ct.c_void_p(dists.data_ptr()),
+                                      _stream(stream)))
+    return (ids, dists, st) if stats else (ids, dists)

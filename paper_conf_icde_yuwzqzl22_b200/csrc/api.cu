@@ -438,6 +438,230 @@ int ganns_build(const float* points, int64_t n, int d, int metric, int degree,
   return GANNS_OK;
 }
 
+// ---------------------------------------------------------------- HNSW
+}  // extern "C"
+
+struct ganns_hnsw {
+  ganns_graph* base = nullptr;          // layer 0, original ids
+  int nlayers = 0;
+  int64_t layer_n[16] = {0};
+  int32_t* upper[16] = {nullptr};       // device, layers 1..nlayers-1, shuffled ids
+  int32_t* perm = nullptr;              // device [n]
+  float* Xp = nullptr;                  // device [layer_n[1]][d], rows of the upper points
+  int d = 0, d_max = 0, metric = 0, device = 0;
+  int32_t entry0 = 0;                   // perm[0]: the entry when there is no upper layer
+};
+
+extern "C" {
+
+void ganns_hnsw_free(ganns_hnsw* h) {
+  if (!h) return;
+  int cur = 0;
+  cudaGetDevice(&cur);
+  cudaSetDevice(h->device);
+  for (auto* p : h->upper) cudaFree(p);
+  cudaFree(h->perm);
+  cudaFree(h->Xp);
+  cudaSetDevice(cur);
+  ganns_graph_free(h->base);
+  delete h;
+}
+
+int ganns_build_hnsw(const float* points, int64_t n, int d, int metric, int degree,
+                     const int8_t* levels_host, const ganns_build_params* p, void* stream,
+                     ganns_hnsw** out) {
+  if (!points || !out || !levels_host) return fail(GANNS_EINVAL, "NULL argument");
+  if (int rc = validate_common(n, d, metric, degree)) return rc;
+  if (!aligned16(points)) return fail(GANNS_EINVAL, "points not 16-byte aligned");
+  const int d_min = p && p->d_min > 0 ? p->d_min : std::max(1, degree / 2);
+  const int l_build = p && p->l_build > 0 ? p->l_build : 64;
+  const int e_build = p && p->e_build > 0 ? p->e_build : l_build;
+  if (d_min > degree || d_min >= n) return fail(GANNS_EINVAL, "bad d_min");
+  if (l_build < d_min || l_build > 1024) return fail(GANNS_EINVAL, "l_build must be in [d_min, 1024]");
+  if (e_build < 1 || e_build > l_build) return fail(GANNS_EINVAL, "e_build must be in [1, l_build]");
+  // (1) shuffled ids: points by level descending, ties by id (stable counting sort)
+  int top = 0;
+  for (int64_t v = 0; v < n; ++v) {
+    if (levels_host[v] < 0 || levels_host[v] >= 16) return fail(GANNS_EINVAL, "level outside [0, 16)");
+    top = std::max(top, int(levels_host[v]));
+  }
+  std::vector<int32_t> perm(static_cast<size_t>(n));
+  std::vector<int64_t> cntl(17, 0);
+  for (int64_t v = 0; v < n; ++v) cntl[levels_host[v]]++;
+  int64_t layer_n[16] = {0};
+  for (int j = top; j >= 0; --j) layer_n[j] = cntl[j] + (j < top ? layer_n[j + 1] : 0);
+  {
+    std::vector<int64_t> pos(17, 0);
+    for (int j = top; j >= 0; --j) pos[j] = (j < top ? pos[j + 1] + cntl[j + 1] : 0);
+    for (int64_t v = 0; v < n; ++v) perm[pos[levels_host[v]]++] = int32_t(v);
+  }
+  ganns_hnsw* h = new (std::nothrow) ganns_hnsw();
+  if (!h) return fail(GANNS_ENOMEM, "host allocation failed");
+  cudaGetDevice(&h->device);
+  h->nlayers = top + 1;
+  h->d = d;
+  h->d_max = degree;
+  h->metric = metric;
+  for (int j = 0; j <= top; ++j) h->layer_n[j] = layer_n[j];
+  h->entry0 = perm[0];
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  float* Xfull = nullptr;
+  int32_t* layer0_shuffled = nullptr;
+  int rc = GANNS_OK;
+  uint64_t tot[4] = {0, 0, 0, 0};
+  auto cleanup = [&](int code) {
+    cudaFree(Xfull);
+    cudaFree(layer0_shuffled);
+    if (code) ganns_hnsw_free(h);
+    return code;
+  };
+  if (cudaMalloc(&h->perm, sizeof(int32_t) * n) != cudaSuccess ||
+      cudaMalloc(&Xfull, sizeof(float) * size_t(n) * d) != cudaSuccess ||
+      cudaMalloc(&layer0_shuffled, sizeof(int32_t) * size_t(n) * degree) != cudaSuccess)
+    return cleanup(fail(GANNS_ENOMEM, "cudaMalloc(hnsw scratch)"));
+  cudaError_t e = cudaMemcpy(h->perm, perm.data(), sizeof(int32_t) * n, cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = launch_gather_rows(points, h->perm, n, d, Xfull, s);
+  if (e != cudaSuccess) return cleanup(cuda_fail(e, "hnsw permute"));
+  // (2) layers top-down, each Algorithm 2 on its prefix
+  UpperLayersHost U;
+  U.top = top;
+  for (int j = top; j >= 0; --j) {
+    int32_t* dst = layer0_shuffled;
+    if (j >= 1) {
+      if (cudaMalloc(&h->upper[j], sizeof(int32_t) * size_t(layer_n[j]) * degree) != cudaSuccess)
+        return cleanup(fail(GANNS_ENOMEM, "cudaMalloc(hnsw layer)"));
+      dst = h->upper[j];
+    }
+    BuildArgs a{};
+    a.X = Xfull;
+    a.n = layer_n[j];
+    a.d = d;
+    a.metric = metric == GANNS_COSINE ? GANNS_IP : metric;
+    a.d_max = degree;
+    a.d_min = d_min;
+    a.l_build = l_build;
+    a.e_build = e_build;
+    int64_t S = p && p->group_size > 0 ? p->group_size : 0;
+    if (S == 0) {
+      double t = 2.0 * std::sqrt(double(std::max<int64_t>(layer_n[j], 1)));
+      int64_t s2 = int64_t(1) << int64_t(std::llround(std::log2(std::max(t, 1.0))));
+      S = std::min<int64_t>(8192, std::max<int64_t>(256, s2));
+    }
+    a.group_size = std::max<int64_t>(1, std::min<int64_t>(S, layer_n[j]));
+    a.max_rounds = -1;
+    a.out_nbr = dst;
+    a.upper = U;
+    a.upper.top = j < top ? top : 0;   // layers above j are finished
+    a.layer = j;
+    rc = run_build(a, s);
+    if (rc) return cleanup(rc);
+    for (int i = 0; i < 4; ++i) tot[i] += a.stats[i];
+    if (j >= 1) {
+      U.nbr[j] = h->upper[j];
+      U.n[j] = layer_n[j];
+    }
+  }
+  // (3) recover the original ids of layer 0
+  ganns_graph* base = nullptr;
+  rc = new_graph(n, d, degree, metric, &base);
+  if (rc) return cleanup(rc);
+  h->base = base;
+  e = launch_relabel(layer0_shuffled, h->perm, n, degree, base->nbr, s);
+  if (e == cudaSuccess && top >= 1) {
+    if (cudaMalloc(&h->Xp, sizeof(float) * size_t(layer_n[1]) * d) != cudaSuccess)
+      return cleanup(fail(GANNS_ENOMEM, "cudaMalloc(hnsw upper rows)"));
+    e = cudaMemcpyAsync(h->Xp, Xfull, sizeof(float) * size_t(layer_n[1]) * d,
+                        cudaMemcpyDeviceToDevice, s);
+  }
+  if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+  if (e != cudaSuccess) return cleanup(cuda_fail(e, "hnsw finalize"));
+  if (p && p->stats)
+    for (int i = 0; i < 4; ++i) p->stats[i] = tot[i];
+  *out = h;
+  return cleanup(GANNS_OK);
+}
+
+int ganns_hnsw_search(const ganns_hnsw* h, const float* points, const float* queries, int64_t nq,
+                      int k, int l, const ganns_search_params* p, int32_t* out_ids,
+                      float* out_dists, void* stream) {
+  if (!h || !h->base) return fail(GANNS_EINVAL, "hnsw is NULL");
+  int e = 0;
+  int32_t entry = 0;
+  if (int rc = validate_search(h->base, points, queries, nq, k, l, p, out_ids, out_dists, &e, &entry))
+    return rc;
+  if (nq == 0) return GANNS_OK;
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  int32_t* entries = nullptr;
+  if (cudaMallocAsync(&entries, sizeof(int32_t) * nq, s) != cudaSuccess)
+    return fail(GANNS_ENOMEM, "cudaMallocAsync(entries)");
+  cudaError_t err = cudaSuccess;
+  if (h->nlayers > 1) {
+    EntryLaunch ea;
+    ea.upper.top = h->nlayers - 1;
+    for (int j = 1; j < h->nlayers; ++j) {
+      ea.upper.nbr[j] = h->upper[j];
+      ea.upper.n[j] = h->layer_n[j];
+    }
+    ea.Xp = h->Xp;
+    ea.np = h->layer_n[1];
+    ea.d = h->d;
+    ea.d_max = h->d_max;
+    ea.metric = h->metric;
+    ea.Q = queries;
+    ea.nq = nq;
+    ea.perm = h->perm;
+    ea.entries = entries;
+    err = launch_entries(ea, s);
+  } else {
+    entry = h->entry0;   // a single layer: every query enters at perm[0]
+    cudaFreeAsync(entries, s);
+    entries = nullptr;
+  }
+  if (err != cudaSuccess) {
+    if (entries) cudaFreeAsync(entries, s);
+    return cuda_fail(err, "hnsw entries");
+  }
+  int32_t* tk = ticket_slot();
+  if (!tk) return fail(GANNS_ENOMEM, "ticket allocation failed");
+  const ganns_graph* g = h->base;
+  SearchLaunch a{g->nbr, points, g->n, g->d, g->d_max, g->metric, queries, nq, k, l, e, entry,
+                 out_ids, out_dists, p ? p->stats : nullptr, tk};
+  a.entries = entries;
+  err = launch_search(a, s);
+  if (entries) cudaFreeAsync(entries, s);
+  return err == cudaSuccess ? GANNS_OK : cuda_fail(err, "hnsw search");
+}
+
+int ganns_hnsw_info(const ganns_hnsw* h, int* nlayers, int64_t* layer_n) {
+  if (!h) return fail(GANNS_EINVAL, "hnsw is NULL");
+  if (nlayers) *nlayers = h->nlayers;
+  if (layer_n)
+    for (int j = 0; j < h->nlayers; ++j) layer_n[j] = h->layer_n[j];
+  return GANNS_OK;
+}
+
+int ganns_hnsw_layer(const ganns_hnsw* h, int layer, int32_t* out_host) {
+  if (!h || !out_host) return fail(GANNS_EINVAL, "NULL argument");
+  if (layer < 0 || layer >= h->nlayers) return fail(GANNS_EINVAL, "layer out of range");
+  if (layer == 0) return ganns_graph_adjacency(h->base, out_host);
+  cudaError_t e = cudaMemcpy(out_host, h->upper[layer], sizeof(int32_t) * size_t(h->layer_n[layer]) * h->d_max,
+                             cudaMemcpyDeviceToHost);
+  return e == cudaSuccess ? GANNS_OK : cuda_fail(e, "cudaMemcpy(layer)");
+}
+
+int ganns_hnsw_perm(const ganns_hnsw* h, int32_t* out_host) {
+  if (!h || !out_host) return fail(GANNS_EINVAL, "NULL argument");
+  cudaError_t e = cudaMemcpy(out_host, h->perm, sizeof(int32_t) * size_t(h->layer_n[0]),
+                             cudaMemcpyDeviceToHost);
+  return e == cudaSuccess ? GANNS_OK : cuda_fail(e, "cudaMemcpy(perm)");
+}
+
+int ganns_hnsw_base(const ganns_hnsw* h, const ganns_graph** base) {
+  if (!h || !base) return fail(GANNS_EINVAL, "NULL argument");
+  *base = h->base;
+  return GANNS_OK;
+}
+
 int ganns_merge_topk(const int32_t* shard_ids, const float* shard_dists, int W, int64_t nq, int k,
                      int32_t* out_ids, float* out_dists, void* stream) {
   if (W < 1 || k < 1 || nq < 0) return fail(GANNS_EINVAL, "bad W / k / nq");

@@ -167,7 +167,7 @@ __global__ void __launch_bounds__(kBuildWarps * 32)
 round_search_kernel(BuildDev B, int64_t lo, int64_t hi, int32_t* __restrict__ Eu,
                     float* __restrict__ Ed, int32_t* __restrict__ indeg,
                     int32_t* __restrict__ touched, int32_t* __restrict__ counters,
-                    const __grid_constant__ CUtensorMap tmap) {
+                    const __grid_constant__ CUtensorMap tmap, const UpperLayers U, int layer) {
   B.g.tmap = &tmap;
   extern __shared__ __align__(128) uint8_t smem[];
   const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -181,9 +181,16 @@ round_search_kernel(BuildDev B, int64_t lo, int64_t hi, int32_t* __restrict__ Eu
   uint64_t* sN = ws.sN;
   uint64_t* sT = ws.sT;
   const int d = B.g.d4 * 4;
-  // line 12: v.N := Search(G_0, v, d_min); G_0 = P_0..P_{i-1}, entry = vertex 0
+  // line 12: v.N := Search(G_0, v, d_min); G_0 = P_0..P_{i-1}, entry = vertex 0;
+  // HNSW: enter through a greedy descent of the finished upper layers,
+  // kept only if the vertex reached is already in G_0 (R-H2)
+  int32_t entry = 0;
+  if (U.top > layer) {
+    const int32_t c = descend<NV4, TPL, L2>(B.g, U, layer + 1, B.g.X + size_t(v) * d, ws);
+    entry = c < lo ? c : 0;
+  }
   SearchStats st;
-  const int cnt = warp_search<NV4, TPL, L2, false>(B.g, B.g.X + size_t(v) * d, 0, B.l_build,
+  const int cnt = warp_search<NV4, TPL, L2, false>(B.g, B.g.X + size_t(v) * d, entry, B.l_build,
                                                    B.e_build, ws, st);
   add_stats(B.stats, st, lane);
   const int dm = B.d_min;
@@ -389,6 +396,12 @@ static int build_t(BuildArgs& a, cudaStream_t s) {
   GANNS_TRY(cudaGetLastError());
 
   // Phase 2 (lines 9-22): merge P_1..P_t into G_0, one round per group
+  UpperLayers U;
+  U.top = a.upper.top;
+  for (int j = 0; j < kMaxLayers; ++j) {
+    U.nbr[j] = a.upper.nbr[j];
+    U.n[j] = a.upper.n[j];
+  }
   int64_t rounds = 0;
   const int64_t last = a.max_rounds < 0 ? ngroups - 1 : std::min<int64_t>(ngroups - 1, a.max_rounds);
   for (int64_t i = 1; i <= last; ++i) {
@@ -397,7 +410,7 @@ static int build_t(BuildArgs& a, cudaStream_t s) {
     GANNS_TRY(cudaMemsetAsync(counters.p, 0, sizeof(int32_t) * 2, s));
     round_search_kernel<NV4, TPL, L2><<<unsigned((nv + kBuildWarps - 1) / kBuildWarps),
                                         kBuildWarps * 32, smem, s>>>(
-        B, lo, hi, Eu.p, Ed.p, indeg.p, touched.p, counters.p, tmap);
+        B, lo, hi, Eu.p, Ed.p, indeg.p, touched.p, counters.p, tmap, U, a.layer);
     const unsigned gs = unsigned(std::min<int64_t>((nslots + 255) / 256, 148 * 4));
     alloc_segments_kernel<<<gs, 256, 0, s>>>(touched.p, indeg.p, segoff.p, counters.p);
     scatter_edges_kernel<<<gs, 256, 0, s>>>(Eu.p, Ed.p, nslots, dm, lo, segoff.p, fill.p, seg.p);

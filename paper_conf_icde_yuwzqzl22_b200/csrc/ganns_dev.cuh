@@ -591,4 +591,33 @@ __device__ int warp_search(const GraphView& g, const float* __restrict__ qrow, i
   return cnt;
 }
 
+// ---------------------------------------------------------------- HNSW
+// Upper layers of an HNSW index (Section IV-D): layer j (1..top) is a
+// graph over the shuffled-id prefix [0, n[j]) of the permuted points.
+constexpr int kMaxLayers = 16;
+struct UpperLayers {
+  int top;                              // highest layer; 0 = no upper layers
+  const int32_t* nbr[kMaxLayers];       // nbr[j], j = 1..top: [n[j]][d_max], shuffled ids
+  int64_t n[kMaxLayers];
+};
+
+// Greedy descent: the GANNS search with l = e = 1 (the best candidate only) from
+// shuffled id 0 through layers top..stop; returns the vertex reached.  `base`
+// carries the permuted points (and their tensor map) and the degree.
+template <int NV4, int TPL, bool L2>
+__device__ int32_t descend(const GraphView& base, const UpperLayers& U, int stop,
+                           const float* __restrict__ q, WarpSmem& ws) {
+  int32_t cur = 0;
+  for (int j = U.top; j >= stop; --j) {
+    GraphView gv = base;
+    gv.nbr = U.nbr[j];
+    gv.n = U.n[j];
+    SearchStats st;
+    warp_search<NV4, TPL, L2, false>(gv, q, cur, 1, 1, ws, st);
+    cur = key_id(unflag(ws.sN[0]));
+    __syncwarp();
+  }
+  return cur;
+}
+
 }  // namespace ganns

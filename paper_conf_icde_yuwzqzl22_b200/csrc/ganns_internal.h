@@ -41,6 +41,12 @@ inline int nv4_for(int d) {
 }
 inline int tpl_for(int d_max) { return d_max <= 32 ? 1 : d_max <= 64 ? 2 : d_max <= 128 ? 4 : -1; }
 
+struct UpperLayersHost {
+  int top = 0;
+  const int32_t* nbr[16] = {nullptr};
+  int64_t n[16] = {0};
+};
+
 struct SearchLaunch {
   const int32_t* nbr;
   const float* X;
@@ -54,7 +60,26 @@ struct SearchLaunch {
   float* out_dists;
   uint32_t* stats;
   int32_t* ticket;      // device scratch counter for the persistent scheduler
+  const int32_t* entries = nullptr;   // per-query entry vertices (HNSW), nullable
 };
+// HNSW: per-query layer-0 entry = perm[greedy descent through the upper layers]
+struct EntryLaunch {
+  UpperLayersHost upper;
+  const float* Xp;      // permuted points, prefix [0, n_1)
+  int64_t np;           // rows of Xp
+  int d, d_max, metric;
+  const float* Q;
+  int64_t nq;
+  const int32_t* perm;
+  int32_t* entries;
+};
+cudaError_t launch_entries(const EntryLaunch& a, cudaStream_t s);
+template <int NV4>
+cudaError_t launch_entries_nv(const EntryLaunch& a, cudaStream_t s);
+cudaError_t launch_gather_rows(const float* X, const int32_t* perm, int64_t n, int d, float* Xp,
+                               cudaStream_t s);
+cudaError_t launch_relabel(const int32_t* in, const int32_t* perm, int64_t n, int d_max,
+                           int32_t* out, cudaStream_t s);
 int32_t* ticket_slot();   // a device int reserved for one launch (ring of slots)
 cudaError_t launch_search(const SearchLaunch& a, cudaStream_t s);
 template <int NV4>
@@ -68,6 +93,8 @@ struct BuildArgs {
   int max_rounds;       // < 0: all
   int32_t* out_nbr;     // device [n][d_max]
   uint64_t stats[4];    // out: iterations, distance computations, searches, rounds
+  UpperLayersHost upper;   // HNSW: finished layers above `layer` (top = 0: plain NSW)
+  int layer = 0;
 };
 int run_build(BuildArgs& a, cudaStream_t s);
 template <int NV4>

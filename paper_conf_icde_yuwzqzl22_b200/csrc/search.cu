@@ -24,6 +24,57 @@ cudaError_t launch_search(const SearchLaunch& a, cudaStream_t s) {
   return cudaErrorInvalidValue;
 }
 
+cudaError_t launch_entries(const EntryLaunch& a, cudaStream_t s) {
+  if (a.nq == 0) return cudaSuccess;
+  switch (nv4_for(a.d)) {
+    case 1: return launch_entries_nv<1>(a, s);
+#ifndef GANNS_DEV_NV1
+    case 2: return launch_entries_nv<2>(a, s);
+    case 4: return launch_entries_nv<4>(a, s);
+    case 8: return launch_entries_nv<8>(a, s);
+#endif
+  }
+  return cudaErrorInvalidValue;
+}
+
+// HNSW bookkeeping: rows of the points in shuffled order, and the
+// relabelling of layer 0 back to the original ids.
+__global__ void gather_rows_kernel(const float4* __restrict__ X, const int32_t* __restrict__ perm,
+                                   int64_t n, int d4, float4* __restrict__ Xp) {
+  for (int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n * d4;
+       i += int64_t(gridDim.x) * blockDim.x) {
+    const int64_t r = i / d4, c = i % d4;
+    Xp[i] = X[size_t(perm[r]) * d4 + c];
+  }
+}
+
+cudaError_t launch_gather_rows(const float* X, const int32_t* perm, int64_t n, int d, float* Xp,
+                               cudaStream_t s) {
+  if (n == 0) return cudaSuccess;
+  gather_rows_kernel<<<148 * 16, 256, 0, s>>>(reinterpret_cast<const float4*>(X), perm, n, d / 4,
+                                              reinterpret_cast<float4*>(Xp));
+  count_launch();
+  return cudaGetLastError();
+}
+
+__global__ void relabel_kernel(const int32_t* __restrict__ in, const int32_t* __restrict__ perm,
+                               int64_t n, int d_max, int32_t* __restrict__ out) {
+  for (int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n * d_max;
+       i += int64_t(gridDim.x) * blockDim.x) {
+    const int64_t r = i / d_max, c = i % d_max;
+    const int32_t u = in[i];
+    out[size_t(perm[r]) * d_max + c] = u >= 0 ? perm[u] : -1;
+  }
+}
+
+cudaError_t launch_relabel(const int32_t* in, const int32_t* perm, int64_t n, int d_max,
+                           int32_t* out, cudaStream_t s) {
+  if (n == 0) return cudaSuccess;
+  relabel_kernel<<<148 * 16, 256, 0, s>>>(in, perm, n, d_max, out);
+  count_launch();
+  return cudaGetLastError();
+}
+
 // ---------------------------------------------------------------- K6
 // Per query, the k smallest (dist, global id) among W sorted shard lists.  One
 // warp per query; each candidate's output position is its rank among all W*k

@@ -19,7 +19,7 @@ __global__ void __launch_bounds__(kSearchWarps * 32, kMinBlocksPerSM)
 search_kernel(GraphView g, const float* __restrict__ Q, int64_t nq, int k, int l, int e,
               int32_t entry, int32_t* __restrict__ out_ids, float* __restrict__ out_dists,
               uint32_t* __restrict__ stats, int32_t* __restrict__ ticket,
-              const __grid_constant__ CUtensorMap tmap) {
+              const int32_t* __restrict__ entries, const __grid_constant__ CUtensorMap tmap) {
   g.tmap = &tmap;
   extern __shared__ __align__(128) uint8_t smem[];
   const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -35,7 +35,8 @@ search_kernel(GraphView g, const float* __restrict__ Q, int64_t nq, int k, int l
   const int64_t q = __shfl_sync(kFull, qt, 0);
   if (q >= nq) break;
   SearchStats st;
-  const int cnt = warp_search<NV4, TPL, L2, false>(g, Q + size_t(q) * (g.d4 * 4), entry, l, e,
+  const int32_t ent = entries != nullptr ? entries[q] : entry;   // HNSW: per-query entry
+  const int cnt = warp_search<NV4, TPL, L2, false>(g, Q + size_t(q) * (g.d4 * 4), ent, l, e,
                                                    ws, st);
   // output: the first k of N, (-1, +inf) padded (R-C8)
   for (int i = lane; i < k; i += 32) {
@@ -91,7 +92,8 @@ static cudaError_t launch_t(const SearchLaunch& a, cudaStream_t s) {
   err = cudaMemsetAsync(a.ticket, 0, sizeof(int32_t), s);
   if (err != cudaSuccess) return err;
   kern<<<dim3(unsigned(blocks)), kSearchWarps * 32, smem, s>>>(
-      g, a.Q, a.nq, a.k, a.l, a.e, a.entry, a.out_ids, a.out_dists, a.stats, a.ticket, tmap);
+      g, a.Q, a.nq, a.k, a.l, a.e, a.entry, a.out_ids, a.out_dists, a.stats, a.ticket, a.entries,
+      tmap);
   count_launch();
   return cudaGetLastError();
 }
@@ -117,5 +119,65 @@ cudaError_t launch_search_nv(const SearchLaunch& a, cudaStream_t s) {
 }
 
 template cudaError_t launch_search_nv<GANNS_NV4>(const SearchLaunch&, cudaStream_t);
+
+// HNSW query entries: one warp per query descends the upper layers
+// greedily (GANNS with l = e = 1 per layer) over the permuted points and writes
+// the layer-0 entry perm[reached vertex].
+template <int NV4, int TPL, bool L2>
+__global__ void __launch_bounds__(kSearchWarps * 32)
+hnsw_entry_kernel(GraphView g, const UpperLayers U, const float* __restrict__ Q, int64_t nq,
+                  const int32_t* __restrict__ perm, int32_t* __restrict__ entries,
+                  const __grid_constant__ CUtensorMap tmap) {
+  extern __shared__ __align__(128) uint8_t smem[];
+  g.tmap = &tmap;
+  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  WarpSmem ws = carve_warp_smem(
+      smem + size_t(w) * warp_smem_bytes(1, TPL, NV4, g.d4, kSearchStageRounds), 1, TPL, NV4, g.d4,
+      kSearchStageRounds);
+  if (lane == 0) mbar_init(ws.mbar, 1);
+  __syncwarp();
+  const int64_t q = int64_t(blockIdx.x) * kSearchWarps + w;
+  if (q >= nq) return;
+  const int32_t c = descend<NV4, TPL, L2>(g, U, 1, Q + size_t(q) * (g.d4 * 4), ws);
+  if (lane == 0) entries[q] = perm[c];
+}
+
+template <int NV4, int TPL, bool L2>
+static cudaError_t entries_t(const EntryLaunch& a, cudaStream_t s) {
+  auto kern = hnsw_entry_kernel<NV4, TPL, L2>;
+  const size_t smem = size_t(kSearchWarps) * warp_smem_bytes(1, TPL, NV4, a.d / 4, kSearchStageRounds);
+  cudaError_t err = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
+  if (err != cudaSuccess) return err;
+  GraphView g{nullptr, a.Xp, nullptr, a.np, a.d_max, a.d / 4, a.metric};
+  CUtensorMap tmap;
+  err = uses_tma(NV4) ? encode_row_tmap(a.Xp, a.np, a.d, &tmap) : zero_tmap(&tmap);
+  if (err != cudaSuccess) return err;
+  UpperLayers U;
+  U.top = a.upper.top;
+  for (int j = 0; j < kMaxLayers; ++j) {
+    U.nbr[j] = a.upper.nbr[j];
+    U.n[j] = a.upper.n[j];
+  }
+  const int64_t blocks = (a.nq + kSearchWarps - 1) / kSearchWarps;
+  kern<<<unsigned(blocks), kSearchWarps * 32, smem, s>>>(g, U, a.Q, a.nq, a.perm, a.entries, tmap);
+  count_launch();
+  return cudaGetLastError();
+}
+
+template <int NV4>
+cudaError_t launch_entries_nv(const EntryLaunch& a, cudaStream_t s) {
+  const bool l2 = a.metric == 0;
+  switch (tpl_for(a.d_max)) {
+    case 1: return l2 ? entries_t<NV4, 1, true>(a, s) : entries_t<NV4, 1, false>(a, s);
+#ifndef GANNS_DEV_ONE
+    case 2: return l2 ? entries_t<NV4, 2, true>(a, s) : entries_t<NV4, 2, false>(a, s);
+    case 4: return l2 ? entries_t<NV4, 4, true>(a, s) : entries_t<NV4, 4, false>(a, s);
+#endif
+  }
+  return cudaErrorInvalidValue;
+}
+
+template cudaError_t launch_entries_nv<GANNS_NV4>(const EntryLaunch&, cudaStream_t);
+
 
 }  // namespace ganns

@@ -1,0 +1,75 @@
+"""HNSW extension (NEXT-1; Section IV-D) on the GPU vs the oracle:
+permutation, layer sizes, every layer's adjacency and the search bit-exact on
+integer-grid data."""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import ganns_synth as syn
+
+pytestmark = pytest.mark.gpu
+if not torch.cuda.is_available():
+    pytest.skip("needs a CUDA device", allow_module_level=True)
+import paper_conf_icde_yuwzqzl22_b200 as g   # noqa: E402
+
+DEV = torch.device("cuda:0")
+
+
+def cu(a):
+    return torch.from_numpy(np.ascontiguousarray(a)).to(DEV)
+
+
+@pytest.mark.parametrize("n,degree,l_build,s,metric,seed", [
+    (3000, 16, 32, 128, "l2", 1),
+    (2500, 32, 64, 256, "l2", 2),
+    (2000, 16, 32, 100, "ip", 3),
+])
+def test_hnsw_build_and_search_parity(n, degree, l_build, s, metric, seed):
+    cfg = syn.with_size(syn.CONFIGS["C1"], n=n, nq=100)
+    X, Q = syn.points(cfg), syn.queries(cfg)
+    if metric == "ip":
+        X, Q = X - 128.0, Q - 128.0
+    levels = syn.hnsw_levels(n, degree // 2, seed)
+    ref = oracle.hnsw_build(X, levels, degree // 2, degree, s, l_build=l_build, metric=metric)
+    idx = g.build_hnsw(cu(X), levels, metric=metric, degree=degree, l_build=l_build, group_size=s)
+    torch.cuda.synchronize()
+    assert idx.nlayers == len(ref["layer_n"]) and idx.layer_n == ref["layer_n"].tolist()
+    assert (idx.perm() == ref["perm"]).all()
+    for j in range(1, idx.nlayers):
+        assert (idx.layer(j) == ref["upper"][j]).all(), j
+    assert (idx.layer(0) == ref["layer0"]).all()
+    ids, dists, st = g.hnsw_search(idx, cu(X), cu(Q), 10, 48, stats=True)
+    oi, od, _, ost = oracle.hnsw_search(ref, X, Q, 10, 48, metric=metric, stats=True)
+    assert (ids.cpu().numpy() == oi).all() and (dists.cpu().numpy() == od).all()
+    st = st.cpu().numpy()
+    assert (st[:, 0] == ost[:, 0]).all() and (st[:, 1] == ost[:, 1]).all()
+
+
+def test_hnsw_theorem_regime():
+    n = 50
+    X = syn.random_int_points(n, 8, 0, 6, 77)
+    levels = np.zeros(n, np.int8)
+    levels[::4] = 1
+    levels[::16] = 2
+    idx = g.build_hnsw(cu(X), levels, degree=64, d_min=4, l_build=n + 1, group_size=7)
+    ref = oracle.hnsw_build(X, levels, 4, 64, 7, l_build=n + 1)
+    for j in range(idx.nlayers):
+        assert (idx.layer(j) == (ref["layer0"] if j == 0 else ref["upper"][j])).all()
+
+
+def test_hnsw_c2_recall_beats_or_matches_nsw():
+    """Full C2 size: HNSW (same degree, d_min, l_build) reaches at least the NSW
+    graph's recall at the same (l, e) and needs fewer layer-0 iterations."""
+    cfg = syn.CONFIGS["C2"]
+    X, Q = syn.points(cfg), syn.queries(cfg)
+    Xd, Qd = cu(X), cu(Q[:2000])
+    levels = syn.hnsw_levels(cfg.n, cfg.degree // 2, 1)
+    idx = g.build_hnsw(Xd, levels, degree=cfg.degree, l_build=64)
+    nsw = g.build(Xd, degree=cfg.degree, l_build=64)
+    gt, _ = oracle.bruteforce(X, Q[:2000], 10)
+    hi, _, hs = g.hnsw_search(idx, Xd, Qd, 10, 64, stats=True)
+    ni, _, ns = g.search(nsw, Xd, Qd, 10, 64, stats=True)
+    rh, rn = oracle.recall(hi.cpu().numpy(), gt), oracle.recall(ni.cpu().numpy(), gt)
+    assert rh >= rn - 0.005, (rh, rn)
+    assert hs[:, 0].float().mean() <= ns[:, 0].float().mean() + 1.0
