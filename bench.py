@@ -114,31 +114,107 @@ class ClockSampler:
                 "reasons": reasons, "samples": len(sm)}
 
 
+SHAPES = {"C1": "SIFT-shaped", "C2": "SIFT1M-shaped", "C3": "GIST1M-shaped",
+          "C4": "GloVe-200-shaped", "C5": "DEEP-shaped"}
+
+
+def workload_name(cfg, kind):
+    return (f"{cfg.name}: {SHAPES[cfg.name]} {cfg.n}x{cfg.d} {cfg.metric}, {kind} degree "
+            f"{cfg.degree}")
+
+
 def make_workload(cfg, rank: int):
     X = syn.points(cfg)
+    if cfg.metric == "cosine":
+        X = syn.normalize_rows(X)   # input preparation: unit rows (Table I "Cosine")
     # every rank draws its own batch of nq queries (weak scaling); rank 0 = the config's
     Qall = syn.queries(cfg, cfg.nq * (rank + 1))
     Q = Qall[rank * cfg.nq:(rank + 1) * cfg.nq]
     return X, np.ascontiguousarray(Q)
 
 
-def ground_truth(torch, Xd, Qd, k):
-    """Exact top-k by (dist, id) with torch fp32 matmuls on the GPU (bench-side
-    measurement only).  Integer-grid data: every term < 2^24, so exact."""
-    torch.backends.cuda.matmul.allow_tf32 = False
+def ground_truth(torch, Xd, Qd, k, metric="l2"):
+    """Exact top-k by (dist, id) on the GPU in fp64 (bench-side measurement only).
+    L2 on integer-grid data: every fp64 term is an exact integer, and the key
+    dist * 2^21 + id (exact below 2^53) breaks ties by id.  IP / cosine (unit
+    rows): ranking by -<q, x>."""
     n = Xd.shape[0]
-    xn = (Xd.double() ** 2).sum(1).float()
-    qn = (Qd.double() ** 2).sum(1).float()
-    best = None
-    shift = 1 << 21
-    for a in range(0, n, 131072):
-        b = min(n, a + 131072)
-        D = qn[:, None] + xn[None, a:b] - 2.0 * (Qd @ Xd[a:b].T)
-        key = D.round().long() * shift + torch.arange(a, b, device=Xd.device)[None, :]
-        kk = torch.topk(key, k, dim=1, largest=False, sorted=True).values
-        best = kk if best is None else torch.topk(torch.cat([best, kk], 1), k, dim=1,
-                                                  largest=False, sorted=True).values
-    return (best % shift).int()
+    Xd64, Qd64 = Xd.double(), Qd.double()
+    best_k = best_i = None
+    shift = float(1 << 21)
+    for a in range(0, n, 65536):
+        b = min(n, a + 65536)
+        dot = Qd64 @ Xd64[a:b].T
+        if metric == "l2":
+            D = (Qd64 ** 2).sum(1)[:, None] + (Xd64[a:b] ** 2).sum(1)[None, :] - 2.0 * dot
+            key = D * shift + torch.arange(a, b, device=Xd.device, dtype=torch.float64)[None, :]
+        else:
+            key = -dot
+        kk, ki = torch.topk(key, k, dim=1, largest=False, sorted=True)
+        ki = ki + a
+        if best_k is None:
+            best_k, best_i = kk, ki
+        else:
+            ck, ci = torch.cat([best_k, kk], 1), torch.cat([best_i, ki], 1)
+            best_k, pos = torch.topk(ck, k, dim=1, largest=False, sorted=True)
+            best_i = torch.gather(ci, 1, pos)
+    return best_i.int()
+
+
+class BenchIndex:
+    """The index a config is benchmarked on: the NSW graph of Algorithm 2, or --
+    for the GloVe-shaped config (BASELINE configs[3]) -- the HNSW-style graph of
+    Section IV-D with seeded levels."""
+
+    def __init__(self, g, cfg, Xd, l_build):
+        self.g, self.cfg, self.Xd = g, cfg, Xd
+        self.hnsw = cfg.name == "C4"
+        if self.hnsw:
+            levels = syn.hnsw_levels(cfg.n, cfg.degree // 2, 1)
+            self.idx = g.build_hnsw(Xd, levels, metric=cfg.metric, degree=cfg.degree,
+                                    l_build=l_build)
+            self.graph = self.idx.base
+            self.build_stats = self.idx.build_stats
+        else:
+            self.idx = None
+            self.graph = g.build(Xd, metric=cfg.metric, degree=cfg.degree, l_build=l_build)
+            self.build_stats = self.graph.build_stats
+        self.kind = "HNSW-style (Section IV-D)" if self.hnsw else "NSW (Algorithm 2)"
+
+    def search(self, Q, k, l, e=0, stats=False, out=None):
+        if self.hnsw:
+            return self.g.hnsw_search(self.idx, self.Xd, Q, k, l, e=e, stats=stats, out=out)
+        return self.g.search(self.graph, self.Xd, Q, k, l, e=e, stats=stats, out=out)
+
+    def search_host(self, torch, Qh, k, l, e, out):
+        """End to end from pinned host buffers through the public API."""
+        if not self.hnsw:
+            return self.g.search_host(self.graph, self.Xd, Qh, k, l, e=e, out=out)
+        Qd = Qh.to(self.Xd.device, non_blocking=True)
+        ids, dists = self.search(Qd, k, l, e=e)
+        out[0].copy_(ids, non_blocking=True)
+        out[1].copy_(dists, non_blocking=True)
+        torch.cuda.current_stream().synchronize()
+        return out
+
+    def oracle_search(self, X, Q, k, l, e, threads):
+        import oracle
+        if not self.hnsw:
+            return oracle.search(self.graph.adjacency(), X, Q, k, l, e=e, metric=self.cfg.metric,
+                                 threads=threads)
+        h = self._oracle_index()
+        ids, dists, _ = oracle.hnsw_search(h, X, Q, k, l, e=e, metric=self.cfg.metric)
+        return ids, dists
+
+    def _oracle_index(self):
+        if not hasattr(self, "_oi"):
+            import numpy as _np
+            ups = {j: self.idx.layer(j) for j in range(1, self.idx.nlayers)}
+            flat = _np.concatenate([ups[j].reshape(-1) for j in range(1, self.idx.nlayers)]) \
+                if ups else _np.zeros(1, _np.int32)
+            self._oi = dict(perm=self.idx.perm(), layer_n=_np.array(self.idx.layer_n, _np.int64),
+                            upper=ups, layer0=self.idx.layer(0), upper_flat=flat)
+        return self._oi
 
 
 def recall_at(ids, gt):
@@ -147,7 +223,7 @@ def recall_at(ids, gt):
     return float(hit) / (k * gt.shape[0])
 
 
-def select_operating_point(torch, g, graph, Xd, Qd, gt, k, target, flush):
+def select_operating_point(torch, index, Qd, gt, k, target, flush):
     """(l, e) sweep: recall@10 of every pair; among the pairs reaching `target`
     the fastest (median of 3 timed launches) is the operating point.  e (explore
     budget) is the paper's fine-grained speed/accuracy knob."""
@@ -159,7 +235,7 @@ def select_operating_point(torch, g, graph, Xd, Qd, gt, k, target, flush):
             flush.zero_()
             a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             a0.record()
-            g.search(graph, Xd, Qd, k, l, e=e)
+            index.search(Qd, k, l, e=e)
             a1.record()
             a1.synchronize()
             ts.append(a0.elapsed_time(a1))
@@ -168,7 +244,7 @@ def select_operating_point(torch, g, graph, Xd, Qd, gt, k, target, flush):
     for l in L_SWEEP:
         best_r = 0.0
         for e in sorted({l, max(k, int(round(0.85 * l))), max(k, int(round(0.7 * l)))}, reverse=True):
-            ids, _ = g.search(graph, Xd, Qd, k, l, e=e)
+            ids, _ = index.search(Qd, k, l, e=e)
             r = recall_at(ids, gt)
             sweep.append((l, e, round(r, 5)))
             best_r = max(best_r, r)
@@ -207,17 +283,17 @@ def run_ours(args):
 
     # ---- GGraphCon build (timed wall clock on device-resident points)
     t0 = time.perf_counter()
-    graph = g.build(Xd, metric=cfg.metric, degree=cfg.degree, l_build=args.l_build)
+    index = BenchIndex(g, cfg, Xd, args.l_build)
     torch.cuda.synchronize()
     build_s = time.perf_counter() - t0
-    b_iters, b_comps, b_searches, b_rounds = graph.build_stats
+    b_iters, b_comps, b_searches, b_rounds = index.build_stats
 
     # ---- (l, e) operating point (see select_operating_point)
-    gt = ground_truth(torch, Xd, Qd, k)
+    gt = ground_truth(torch, Xd, Qd, k, cfg.metric)
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
-    l_star, e_star, sweep, chosen = select_operating_point(torch, g, graph, Xd, Qd, gt, k,
-                                                           args.target, flush)
-    ids, dists, st = g.search(graph, Xd, Qd, k, l_star, e=e_star, stats=True)
+    l_star, e_star, sweep, chosen = select_operating_point(torch, index, Qd, gt, k, args.target,
+                                                           flush)
+    ids, dists, st = index.search(Qd, k, l_star, e=e_star, stats=True)
     rec = recall_at(ids, gt)
     st = st.long()
     d = cfg.d
@@ -233,7 +309,7 @@ def run_ours(args):
     out = (torch.empty((Q.shape[0], k), dtype=torch.int32, device=dev),
            torch.empty((Q.shape[0], k), dtype=torch.float32, device=dev))
     for _ in range(args.warmup):
-        g.search(graph, Xd, Qd, k, l_star, e=e_star, out=out)
+        index.search(Qd, k, l_star, e=e_star, out=out)
     torch.cuda.synchronize()
     launches0 = g.kernel_launches()
     times = []
@@ -246,7 +322,7 @@ def run_ours(args):
             e0 = torch.cuda.Event(enable_timing=True)
             e1 = torch.cuda.Event(enable_timing=True)
             e0.record(stream)
-            g.search(graph, Xd, Qd, k, l_star, e=e_star, out=out)
+            index.search(Qd, k, l_star, e=e_star, out=out)
             e1.record(stream)
             e1.synchronize()
             times.append(e0.elapsed_time(e1))
@@ -269,13 +345,13 @@ def run_ours(args):
     hout = (torch.empty((Q.shape[0], k), dtype=torch.int32).pin_memory(),
             torch.empty((Q.shape[0], k), dtype=torch.float32).pin_memory())
     for _ in range(2):
-        g.search_host(graph, Xd, Qh, k, l_star, e=e_star, out=hout)
+        index.search_host(torch, Qh, k, l_star, e_star, hout)
     e2e_times = []
     for _ in range(args.steps):
         flush.zero_()
         torch.cuda.synchronize()
         t0 = time.perf_counter()
-        g.search_host(graph, Xd, Qh, k, l_star, e=e_star, out=hout)
+        index.search_host(torch, Qh, k, l_star, e_star, hout)
         e2e_times.append(time.perf_counter() - t0)
     e2e_t = torch.tensor([sum(e2e_times)], dtype=torch.float64, device=dev)
     if world > 1:
@@ -305,8 +381,7 @@ def run_ours(args):
         "vs_baseline": None,
         "dtype": "f32",
         "data": "synthetic",
-        "config": {"workload": f"{args.config}: SIFT1M-shaped {cfg.n}x{cfg.d} L2, NSW degree "
-                               f"{cfg.degree}, {Q.shape[0]} queries/GPU, k={k}",
+        "config": {"workload": workload_name(cfg, index.kind) + f", {Q.shape[0]} queries/GPU, k={k}",
                    "l": l_star, "e": e_star, "recall_at_10": round(rec, 5),
                    "selection": "fastest (l, e) with recall@10 >= target among the sweep",
                    "le_for_recall": {str(t): chosen.get(t) for t in (0.9, 0.95, 0.99)},
@@ -325,12 +400,11 @@ def run_ours(args):
         "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak,
                      "unit": "GB/s", "frac": round(achieved / peak, 4), "traffic": traffic,
                      "peak_kind": peak_kind, "alg_bytes_per_launch": alg_bytes,
-                     "kernel": "ganns::search_kernel<1,1,true>"},
+                     "kernel": f"ganns::search_kernel (d={cfg.d}, d_max={cfg.degree}, {cfg.metric})"},
         "clocks": clk.summary(),
     }
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        line["cpu_baseline"] = cpu_baseline(graph.adjacency(), X, Q, k, l_star, e_star,
-                                            args.cpu_seconds)
+        line["cpu_baseline"] = cpu_baseline(index, X, Q, k, l_star, e_star, args.cpu_seconds)
     if rank == 0:
         s = json.dumps(line)
         print(s, flush=True)
@@ -341,18 +415,18 @@ def run_ours(args):
         dist.destroy_process_group()
 
 
-def cpu_baseline(nbr, X, Q, k, l, e, seconds):
+def cpu_baseline(index, X, Q, k, l, e, seconds):
     """The oracle's search (plain C, one pthread per host core) on a bounded sample
     of the same queries and graph.  Returns the cpu_baseline object."""
     import oracle
     cores = oracle.ncores()
     m = 64
     t0 = time.perf_counter()
-    oracle.search(nbr, X, Q[:m], k, l, e=e, threads=cores)
+    index.oracle_search(X, Q[:m], k, l, e, cores)
     dt = time.perf_counter() - t0
     m2 = int(min(len(Q), max(m, m * seconds / max(dt, 1e-3))))
     t0 = time.perf_counter()
-    oracle.search(nbr, X, Q[:m2], k, l, e=e, threads=cores)
+    index.oracle_search(X, Q[:m2], k, l, e, cores)
     dt = time.perf_counter() - t0
     return {"value": round(m2 / dt, 1), "unit": "queries/s", "cores": cores, "kind": "oracle",
             "sample": f"first {m2} of the {len(Q)} queries, same graph, l={l}, e={e}, {dt:.1f} s"}
@@ -370,28 +444,29 @@ def run_reference(args):
     cfg = syn.CONFIGS[args.config]
     k = cfg.k
     X, Q = make_workload(cfg, 0)
-    # index set-up (not timed): the graph the GPU arm searches, deterministic
+    # index set-up (not timed): the graph the GPU arm searches (deterministic) and
+    # the same (l, e) operating point
     Xd = torch.from_numpy(X).cuda()
-    graph = g.build(Xd, metric=cfg.metric, degree=cfg.degree, l_build=args.l_build)
-    nbr = graph.adjacency()
+    index = BenchIndex(g, cfg, Xd, args.l_build)
     Qd = torch.from_numpy(Q).cuda()
-    gt = ground_truth(torch, Xd, Qd, k)
+    gt = ground_truth(torch, Xd, Qd, k, cfg.metric)
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=Xd.device)
-    l_star, e_star, _, _ = select_operating_point(torch, g, graph, Xd, Qd, gt, k, args.target, flush)
-    del Xd, Qd
+    l_star, e_star, _, _ = select_operating_point(torch, index, Qd, gt, k, args.target, flush)
+    index.oracle_search(X, Q[:2], k, l_star, e_star, 1)   # materialise the host copy
+    del Qd, flush
     cores = oracle.ncores()
     per_step = 48
     for _ in range(args.warmup):
-        oracle.search(nbr, X, Q[:16], k, l_star, e=e_star, threads=cores)
+        index.oracle_search(X, Q[:16], k, l_star, e_star, cores)
     t0 = time.perf_counter()
-    oracle.search(nbr, X, Q[:per_step], k, l_star, e=e_star, threads=cores)
+    index.oracle_search(X, Q[:per_step], k, l_star, e_star, cores)
     dt = time.perf_counter() - t0
     per_step = int(max(cores, min(len(Q), per_step * 6.0 / max(dt, 1e-3))))
     times = []
     for s in range(args.steps):
         a = (s * per_step) % max(1, len(Q) - per_step)
         t0 = time.perf_counter()
-        oracle.search(nbr, X, Q[a:a + per_step], k, l_star, e=e_star, threads=cores)
+        index.oracle_search(X, Q[a:a + per_step], k, l_star, e_star, cores)
         times.append(time.perf_counter() - t0)
     tot = sum(times)
     v = per_step * args.steps / tot
@@ -402,8 +477,8 @@ def run_reference(args):
         "unit": "queries/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
         "ms_per_step": round(tot / args.steps * 1e3, 3), "higher_is_better": True,
         "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-        "config": {"workload": f"{args.config}: SIFT1M-shaped {cfg.n}x{cfg.d} L2, NSW degree "
-                               f"{cfg.degree}, k={k}", "l": l_star, "e": e_star},
+        "config": {"workload": workload_name(cfg, index.kind) + f", k={k}", "l": l_star,
+                   "e": e_star},
         "cpu_baseline": {"value": round(v, 1), "unit": "queries/s", "cores": cores,
                          "kind": "oracle", "sample": sample},
         "e2e": {"value": round(v, 1), "unit": "queries/s", "h2d_bytes_per_step": 0,

@@ -45,7 +45,7 @@ class Config:
 CONFIGS = {
     "C1": Config("C1", 1, 10_000, 128, 0, 255, 32, 0.25, 16, 0.03, "l2", 100, 16),
     "C2": Config("C2", 2, 1_000_000, 128, 0, 255, 32, 0.25, 16, 0.03, "l2", 10_000, 32),
-    "C3": Config("C3", 3, 1_000_000, 960, 0, 127, 32, 0.25, 32, 0.03, "l2", 1_000, 32),
+    "C3": Config("C3", 3, 1_000_000, 960, 0, 127, 32, 0.25, 20, 0.03, "l2", 1_000, 32),
     "C4": Config("C4", 4, 1_183_514, 200, -127, 127, 256, 0.25, 24, 0.03, "cosine", 10_000, 32,
                  zipf=1.1),
     "C5": Config("C5", 5, 100_000_000, 96, -127, 127, 1024, 0.25, 16, 0.03, "l2", 10_000, 32,

@@ -142,14 +142,17 @@ struct SearchStats {
 
 // Per-warp shared memory: [stage: 32 vector rows, TMA destination][N][T][mbar][bitmap]
 __host__ __device__ constexpr int lpad32(int l) { return (l + 31) & ~31; }
+// uses_tma: the tile::gather4 tensor map is used (d <= 256: the map's box is one
+// row of <= 256 elements); wider rows are staged with 1-D bulk copies.
 __host__ __device__ constexpr bool uses_tma(int nv4) { return nv4 <= 2; }
+constexpr int kWideStageRows = 8;   // d > 256: rows per TMA round (4 rounds per exploration)
 // The <= 32 rows of one exploration are staged in `rounds` TMA rounds (1 or 2):
 // 2 rounds halve the stage (more resident warps, the throughput-bound batched
 // search); 1 round saves a memory round trip (the latency-bound build).
 constexpr int kSearchStageRounds = 2;
 constexpr int kBuildStageRounds = 1;
 __host__ __device__ constexpr size_t stage_bytes(int nv4, int d4, int rounds) {
-  return uses_tma(nv4) ? size_t(32 / rounds) * d4 * 16 : 0;
+  return uses_tma(nv4) ? size_t(32 / rounds) * d4 * 16 : size_t(kWideStageRows) * d4 * 16;
 }
 __host__ __device__ constexpr size_t warp_smem_bytes(int l, int tpl, int nv4, int d4, int rounds) {
   // rounded to 128 B: the stage (first) must be 128-B aligned for tensor TMA
@@ -307,39 +310,47 @@ __device__ __forceinline__ float tma_dot(const GraphView& g, const float4 (&qv)[
   return p[0];
 }
 
-// Whole-warp form (S = 32, d > 256): rows in batches of B, a transposing
-// butterfly over the top log2(B) lane bits, plain reduction over the rest.
+// Whole-warp form (S = 32, d > 256): rows are staged kWideStageRows at a time by
+// 1-D TMA bulk copies (one per row, issued by the lane owning the neighbour);
+// each lane reads float4 columns lane + 32f of every staged row from shared
+// memory; per round a transposing butterfly over the top 3 lane bits and a plain
+// reduction over the rest leave lane j with row j's total.
 template <int C, bool L2, bool FULL>
-__device__ __forceinline__ float warp_dot(const GraphView& g, const float4 (&qv)[C],
-                                          int32_t u_mine, int lane) {
-  constexpr int B = C >= 8 ? 1 : 8 / C;
-  constexpr int LOGB = B == 8 ? 3 : B == 4 ? 2 : B == 2 ? 1 : 0;
-  const char* base = reinterpret_cast<const char*>(g.X) + lane * 16;
+__device__ __forceinline__ float wide_dot(const GraphView& g, const float4 (&qv)[C],
+                                          int32_t u_mine, int lane, WarpSmem& ws) {
+  constexpr int R = kWideStageRows;   // 8 rows per round, 4 rounds
   const uint32_t rowbytes = uint32_t(g.d4) * 16u;
-  const int32_t u_safe = u_mine < 0 ? 0 : u_mine;
-  int coff[C];
-#pragma unroll
-  for (int f = 0; f < C; ++f) coff[f] = (FULL || lane + 32 * f < g.d4) ? 32 * f : g.d4 - 1 - lane;
   float dres = 0.f;
+#pragma unroll 1
+  for (int r = 0; r < 32 / R; ++r) {
+    const bool mine = u_mine >= 0 && (lane / R) == r;
+    const unsigned vm = __ballot_sync(kFull, mine);
+    if (vm) {
+      __syncwarp();
+      fence_proxy_async_smem();
+      if (lane == 0) mbar_arrive_expect_tx(ws.mbar, uint32_t(__popc(vm)) * rowbytes);
+      __syncwarp();
+      if (mine)
+        tma_row(reinterpret_cast<char*>(ws.stage) + size_t(lane % R) * rowbytes,
+                reinterpret_cast<const char*>(g.X) + uint64_t(uint32_t(u_mine)) * rowbytes,
+                rowbytes, ws.mbar);
+      mbar_wait(ws.mbar, ws.phase);
+      ws.phase ^= 1u;
+    }
+    float p[R];
 #pragma unroll
-  for (int b = 0; b < 32 / B; ++b) {
-    float p[B];
-#pragma unroll
-    for (int i = 0; i < B; ++i) {
-      const int32_t u = __shfl_sync(kFull, u_safe, b * B + i);
-      const float4* rp = reinterpret_cast<const float4*>(base + uint64_t(uint32_t(u)) * rowbytes);
-      float4 x[C];
-#pragma unroll
-      for (int f = 0; f < C; ++f) x[f] = ldg_stream(rp + coff[f]);
+    for (int i = 0; i < R; ++i) {
+      const float4* rp = ws.stage + size_t(i) * g.d4;
       uint64_t acc = 0;
 #pragma unroll
       for (int f = 0; f < C; ++f)
-        if (FULL || lane + 32 * f < g.d4) acc = accum4<L2>(acc, qv[f], x[f]);
+        if (FULL || lane + 32 * f < g.d4) acc = accum4<L2>(acc, qv[f], rp[lane + 32 * f]);
       p[i] = hsum2(acc);
     }
+    // transposing butterfly over lane bits 4,3,2 (8 rows), then bits 1,0
 #pragma unroll
-    for (int s = 0; s < LOGB; ++s) {
-      const int half = B >> (s + 1), off = 16 >> s;
+    for (int st = 0; st < 3; ++st) {
+      const int half = R >> (st + 1), off = 16 >> st;
       const bool up = lane & off;
 #pragma unroll
       for (int i = 0; i < half; ++i) {
@@ -348,10 +359,11 @@ __device__ __forceinline__ float warp_dot(const GraphView& g, const float4 (&qv)
         p[i] = keep + __shfl_xor_sync(kFull, send, off);
       }
     }
-#pragma unroll
-    for (int off = 16 >> LOGB; off >= 1; off >>= 1) p[0] += __shfl_xor_sync(kFull, p[0], off);
-    float got = __shfl_sync(kFull, p[0], (lane & (B - 1)) << (5 - LOGB));
-    if ((lane >> LOGB) == b) dres = got;
+    p[0] += __shfl_xor_sync(kFull, p[0], 2);
+    p[0] += __shfl_xor_sync(kFull, p[0], 1);
+    // lane L holds the total of row (L >> 2) of this round
+    const float got = __shfl_sync(kFull, p[0], (lane % R) << 2);
+    if (lane / R == r) dres = got;
   }
   return dres;
 }
@@ -362,7 +374,7 @@ __device__ __forceinline__ float group_distances(const GraphView& g,
                                                  int32_t u_mine, float cbase, float qinv,
                                                  int lane, WarpSmem& ws) {
   constexpr int S = VecLayout<NV4>::S, C = VecLayout<NV4>::C;
-  static_assert(uses_tma(NV4) == (S < 32), "TMA staging is used exactly for the segment form");
+  static_assert(uses_tma(NV4) == (S < 32), "tile::gather4 is used exactly for the segment form");
   const bool full = g.d4 == S * C;
   float dot;
   if constexpr (S < 32) {
@@ -373,8 +385,8 @@ __device__ __forceinline__ float group_distances(const GraphView& g,
       dot = full ? tma_dot<S, C, L2, true, 2>(g, qv, u_mine, lane, ws)
                  : tma_dot<S, C, L2, false, 2>(g, qv, u_mine, lane, ws);
   } else {
-    dot = full ? warp_dot<C, L2, true>(g, qv, u_mine, lane)
-               : warp_dot<C, L2, false>(g, qv, u_mine, lane);
+    dot = full ? wide_dot<C, L2, true>(g, qv, u_mine, lane, ws)
+               : wide_dot<C, L2, false>(g, qv, u_mine, lane, ws);
   }
   if constexpr (L2) return dot;
   else return cbase - dot * qinv;   // IP: 0 - dot (exact); COSINE: 1 - dot/||q||
@@ -473,9 +485,11 @@ __device__ int warp_search(const GraphView& g, const float* __restrict__ qrow, i
     spec_v = w;
     // (3) bulk distance computation
     if constexpr (!uses_tma(NV4)) {
+      // wide rows are staged in 4 rounds: warm all of them in L2 at once so the
+      // later rounds find their lines close
 #pragma unroll
       for (int t = 0; t < TPL; ++t)
-        if (u[t] >= 0)
+        if (u[t] >= 0 && (lane / kWideStageRows) != 0)
           prefetch_row_l2(g.X + size_t(u[t]) * (g.d4 * 4), uint32_t(g.d4) * 16u);
     }
     uint64_t key[TPL];
