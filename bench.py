@@ -269,8 +269,10 @@ def run_ours(args):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
-    if world > 1:
-        dist.init_process_group("nccl")
+    distributed = "RANK" in os.environ          # launched by torchrun (any world size)
+    if distributed:
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     cfg = syn.CONFIGS[args.config]
@@ -313,7 +315,7 @@ def run_ours(args):
     torch.cuda.synchronize()
     launches0 = g.kernel_launches()
     times = []
-    if world > 1:
+    if distributed:
         dist.barrier()
     torch.cuda.synchronize()
     with ClockSampler(local) as clk:
@@ -327,12 +329,12 @@ def run_ours(args):
             e1.synchronize()
             times.append(e0.elapsed_time(e1))
     torch.cuda.synchronize()
-    if world > 1:
+    if distributed:
         dist.barrier()
     launches = g.kernel_launches() - launches0
     t_total = sum(times) / 1e3
     t_max = torch.tensor([t_total], dtype=torch.float64, device=dev)
-    if world > 1:
+    if distributed:
         dist.all_reduce(t_max, op=dist.ReduceOp.MAX)
     t_total = float(t_max.item())
     total_queries = Q.shape[0] * args.steps * world
@@ -354,7 +356,7 @@ def run_ours(args):
         index.search_host(torch, Qh, k, l_star, e_star, hout)
         e2e_times.append(time.perf_counter() - t0)
     e2e_t = torch.tensor([sum(e2e_times)], dtype=torch.float64, device=dev)
-    if world > 1:
+    if distributed:
         dist.all_reduce(e2e_t, op=dist.ReduceOp.MAX)
     e2e_qps = total_queries / float(e2e_t.item())
 
@@ -411,7 +413,8 @@ def run_ours(args):
         if args.json_out:
             with open(args.json_out, "w") as f:
                 f.write(s + "\n")
-    if world > 1:
+    if distributed:
+        dist.barrier()
         dist.destroy_process_group()
 
 
