@@ -149,7 +149,10 @@ constexpr int kWideStageRows = 8;   // d > 256: rows per TMA round (4 rounds per
 // The <= 32 rows of one exploration are staged in `rounds` TMA rounds (1 or 2):
 // 2 rounds halve the stage (more resident warps, the throughput-bound batched
 // search); 1 round saves a memory round trip (the latency-bound build).
-constexpr int kSearchStageRounds = 2;
+#ifndef GANNS_SEARCH_ROUNDS
+#define GANNS_SEARCH_ROUNDS 2
+#endif
+constexpr int kSearchStageRounds = GANNS_SEARCH_ROUNDS;
 constexpr int kBuildStageRounds = 1;
 __host__ __device__ constexpr size_t stage_bytes(int nv4, int d4, int rounds) {
   return uses_tma(nv4) ? size_t(32 / rounds) * d4 * 16 : size_t(kWideStageRows) * d4 * 16;
@@ -257,10 +260,20 @@ __device__ __forceinline__ float tma_dot(const GraphView& g, const float4 (&qv)[
     // copy per row.
     const bool g4 = (g.d4 & 1) == 0;
     const int32_t uo = u_mine >= 0 ? u_mine : 0x7fffffff;
-    const int32_t u1 = __shfl_down_sync(kFull, uo, 1);
-    const int32_t u2 = __shfl_down_sync(kFull, uo, 2);
-    const int32_t u3 = __shfl_down_sync(kFull, uo, 3);
-    const bool issuer = g4 ? ((lane & 3) == 0 && my_round == r && (uo & u1 & u2 & u3) != 0x7fffffff)
+    // rows of stage slots my_slot+1..+3 of this round: with >= 4 passes per round
+    // they belong to the next 3 lanes; otherwise to lane r*PPR + k%PPR + S*(k/PPR)
+    int32_t u1, u2, u3;
+    if constexpr (PPR % 4 == 0) {
+      u1 = __shfl_down_sync(kFull, uo, 1);
+      u2 = __shfl_down_sync(kFull, uo, 2);
+      u3 = __shfl_down_sync(kFull, uo, 3);
+    } else {
+      auto lane_of = [r](int k) { return r * PPR + k % PPR + S * (k / PPR); };
+      u1 = __shfl_sync(kFull, uo, lane_of((my_slot + 1) & 31));
+      u2 = __shfl_sync(kFull, uo, lane_of((my_slot + 2) & 31));
+      u3 = __shfl_sync(kFull, uo, lane_of((my_slot + 3) & 31));
+    }
+    const bool issuer = g4 ? ((my_slot & 3) == 0 && my_round == r && (uo & u1 & u2 & u3) != 0x7fffffff)
                            : (u_mine >= 0 && my_round == r);
     const unsigned vm = __ballot_sync(kFull, issuer);
     if (vm) {
@@ -381,6 +394,11 @@ __device__ __forceinline__ float group_distances(const GraphView& g,
     if (ws.rounds == 1)
       dot = full ? tma_dot<S, C, L2, true, 1>(g, qv, u_mine, lane, ws)
                  : tma_dot<S, C, L2, false, 1>(g, qv, u_mine, lane, ws);
+#if GANNS_SEARCH_ROUNDS == 4
+    else if (ws.rounds == 4)
+      dot = full ? tma_dot<S, C, L2, true, 4>(g, qv, u_mine, lane, ws)
+                 : tma_dot<S, C, L2, false, 4>(g, qv, u_mine, lane, ws);
+#endif
     else
       dot = full ? tma_dot<S, C, L2, true, 2>(g, qv, u_mine, lane, ws)
                  : tma_dot<S, C, L2, false, 2>(g, qv, u_mine, lane, ws);
