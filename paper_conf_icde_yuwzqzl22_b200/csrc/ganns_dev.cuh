@@ -486,6 +486,7 @@ __device__ int warp_search(const GraphView& g, const float* __restrict__ qrow, i
       }
     }
     if (found < 0) break;
+    __syncwarp();   // the explored mark (one lane's store) is visible to the whole warp
     st.iters++;
     // (2) neighbourhood exploration: T <- out-neighbours of v
     int32_t u[TPL];
