@@ -53,6 +53,8 @@ def lib():
         _lib.ora_alg2.argtypes = [P, i64, i32, i32, i32, i32, i32, i32, i64, i32, i32, P, P, P]
         _lib.ora_naive_parallel.argtypes = [P, i64, i32, i32, i32, i32, i32, i32, i64, P, P]
         _lib.ora_merge_topk.argtypes = [P, P, i32, i64, i32, P, P]
+        _lib.ora_knn_descent.argtypes = [P, i64, i32, i32, i32, P, i32, P, P, P]
+        _lib.ora_knn_descent.restype = ct.c_int
         _lib.ora_hnsw_build.argtypes = [P, i64, i32, i32, P, i32, i32, i32, i32, i64, P, P, P,
                                         P, P]
         _lib.ora_hnsw_search.argtypes = [P, P, i32, P, P, i64, i32, P, i32, i32, P, i64, i32,
@@ -247,3 +249,19 @@ def hnsw_search(h, X, Q, k, l, e=0, metric="l2", stats=False):
                                  layer0.shape[1], _p(X), X.shape[1], METRICS[metric], _p(Q), nq,
                                  k, l, e, _p(ids), _p(dists), _p(st), _p(ent)))
     return (ids, dists, ent, st) if stats else (ids, dists, ent)
+
+
+def knn_descent(X, init, K, max_iters=30, metric="l2"):
+    """KNN graph by neighbours-of-neighbours iterations.
+    Returns (ids [n,K], dists [n,K], iterations, changed_in_last_iteration)."""
+    X = _f32(X)
+    init = _i32(init)
+    n = X.shape[0]
+    ids = np.full((n, K), -1, np.int32)
+    dists = np.empty((n, K), np.float32)
+    ch = ct.c_int64()
+    it = lib().ora_knn_descent(_p(X), n, X.shape[1], METRICS[metric], K, _p(init), max_iters,
+                               _p(ids), _p(dists), ct.byref(ch))
+    if it < 0:
+        raise ValueError(f"oracle returned {it}")
+    return ids, dists, it, ch.value

@@ -369,3 +369,48 @@ def test_hnsw_quality_at_least_nsw():
     ih, _, _ = oracle.hnsw_search(h, X, Q, 10, 32)
     inn, _ = oracle.search(nsw, X, Q, 10, 32)
     assert oracle.recall(ih, gt) >= oracle.recall(inn, gt) - 0.02
+
+
+# --------------------------------------- KNN graph, NN-Descent form (NEXT-4)
+def _exact_knn_lists(X, K):
+    gi, gd = oracle.bruteforce(X, X, K + 1)
+    ids = np.array([[u for u in r if u != i][:K] for i, r in enumerate(gi)], np.int32)
+    return ids
+
+
+def test_knn_exact_init_is_a_fixed_point():
+    """If every list already holds the exact K nearest, no proposal can enter:
+    one iteration, nothing changes ("terminates when ... cease to change")."""
+    X = syn.random_int_points(300, 6, 0, 50, 4)
+    ex = _exact_knn_lists(X, 8)
+    ids, dists, it, ch = oracle.knn_descent(X, ex, 8, 10)
+    assert it == 1 and ch == 0
+    assert (ids == ex).all()
+
+
+def test_knn_lists_only_improve_and_converge():
+    cfg = syn.with_size(syn.CONFIGS["C1"], n=1200)
+    X = syn.points(cfg)
+    init = syn.random_graph(len(X), 12, seed=9)
+    prev = None
+    for t in range(0, 6):
+        ids, dists, it, ch = oracle.knn_descent(X, init, 12, t)
+        if prev is not None:
+            assert (dists <= prev + 0).all()          # element-wise non-increasing
+        prev = dists
+        for v in range(0, len(X), 97):              # rows sorted, distinct, no self loop
+            row = ids[v][ids[v] >= 0]
+            assert v not in row and len(set(row.tolist())) == len(row)
+            assert all(dists[v][i] <= dists[v][i + 1] for i in range(len(row) - 1))
+            assert dists[v][0] == oracle.distance(X[v], X[row[0]])
+    ids, dists, it, ch = oracle.knn_descent(X, init, 12, 50)
+    assert ch == 0 and it < 50
+    assert oracle.recall(ids, _exact_knn_lists(X, 12)) > 0.9
+
+
+def test_knn_complete_lists_are_exact():
+    """K = n - 1: every list holds all other points, sorted = the exact lists."""
+    X = syn.random_int_points(20, 3, 0, 9, 6)
+    init = syn.random_graph(20, 19, seed=1)
+    ids, dists, it, ch = oracle.knn_descent(X, init, 19, 3)
+    assert (ids == _exact_knn_lists(X, 19)).all()
