@@ -205,6 +205,22 @@ GANNS_API int ganns_hnsw_base(const ganns_hnsw *h, const ganns_graph **base);
 /* ganns_hnsw_free -- NULL is a no-op. */
 GANNS_API void ganns_hnsw_free(ganns_hnsw *h);
 
+/* ---------------------------------------------------------------- KNN graph
+ * ganns_build_knn -- KNN graph (every list = K nearest, k = d_min = d_max)
+ * by neighbours-of-neighbours iterations (Section IV-D, after
+ * NN-Descent [9]): from the random lists init_host, each iteration joins every
+ * pair of a vertex's neighbours (its list and its reverse list, capped at the K
+ * nearest) and every list keeps its K nearest distinct candidates; stops when no
+ * list changes or after max_iters iterations.
+ *   init_host   host int32 [n][K]: distinct ids != row, no -1 (e.g. random)
+ *   K           1 <= K <= 32, K < n
+ *   out         graph [n][K] ascending by (dist, id); iters_out / changed_last
+ *               (nullable): iterations run, lists changed in the last one.
+ * Proposal buffer: n * 2K * (2K - 1) entries of 12 bytes (ENOMEM if it does not fit). Syncs. */
+GANNS_API int ganns_build_knn(const float *points, int64_t n, int d, int metric, int K,
+                              const int32_t *init_host, int max_iters, void *stream,
+                              ganns_graph **out, int *iters_out, int64_t *changed_last);
+
 /* ganns_last_error -- thread-local message of the last failing call ("" if none). */
 GANNS_API const char *ganns_last_error(void);
 

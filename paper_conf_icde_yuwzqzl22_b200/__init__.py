@@ -61,6 +61,8 @@ def _load():
         "ganns_hnsw_layer": [P, i32, P],
         "ganns_hnsw_perm": [P, P],
         "ganns_hnsw_base": [P, ct.POINTER(P)],
+        "ganns_build_knn": [P, i64, i32, i32, i32, P, i32, P, ct.POINTER(P), ct.POINTER(i32),
+                            ct.POINTER(i64)],
     }
     for name, args in sig.items():
         f = getattr(lib, name)
@@ -86,7 +88,7 @@ ABI_SYMBOLS = ("ganns_build", "ganns_search", "ganns_search_ex", "ganns_search_h
                "ganns_graph_save", "ganns_graph_load", "ganns_graph_free", "ganns_last_error",
                "ganns_kernel_launches", "ganns_build_hnsw", "ganns_hnsw_search",
                "ganns_hnsw_info", "ganns_hnsw_layer", "ganns_hnsw_perm", "ganns_hnsw_base",
-               "ganns_hnsw_free")
+               "ganns_hnsw_free", "ganns_build_knn")
 
 
 def lib():
@@ -337,3 +339,20 @@ def hnsw_search(index: Hnsw, points: torch.Tensor, queries: torch.Tensor, k: int
                                       ct.c_void_p(ids.data_ptr()), ct.c_void_p(dists.data_ptr()),
                                       _stream(stream)))
     return (ids, dists, st) if stats else (ids, dists)
+
+
+def build_knn(points: torch.Tensor, init: np.ndarray, K: int, metric: str = "l2",
+              max_iters: int = 30, stream=None):
+    """KNN graph by neighbours-of-neighbours iterations.  `init` int32
+    [n, K] random lists (e.g. ganns_synth.random_graph(n, K, seed)).  Returns
+    (Graph, iterations, lists changed in the last iteration)."""
+    points = _dev_f32(points, "points")
+    init = np.ascontiguousarray(init, dtype=np.int32)
+    h = ct.c_void_p()
+    it, ch = ct.c_int(), ct.c_int64()
+    with torch.cuda.device(points.device):
+        _check(_lib.ganns_build_knn(ct.c_void_p(points.data_ptr()), points.shape[0],
+                                    points.shape[1], METRICS[metric], K,
+                                    init.ctypes.data_as(ct.c_void_p), max_iters, _stream(stream),
+                                    ct.byref(h), ct.byref(it), ct.byref(ch)))
+    return Graph(h), it.value, ch.value

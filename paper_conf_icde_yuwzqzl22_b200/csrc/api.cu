@@ -662,6 +662,49 @@ int ganns_hnsw_base(const ganns_hnsw* h, const ganns_graph** base) {
   return GANNS_OK;
 }
 
+int ganns_build_knn(const float* points, int64_t n, int d, int metric, int K,
+                    const int32_t* init_host, int max_iters, void* stream, ganns_graph** out,
+                    int* iters_out, int64_t* changed_last) {
+  if (!points || !init_host || !out) return fail(GANNS_EINVAL, "NULL argument");
+  if (int rc = validate_common(n, d, metric, 2)) return rc;
+  if (K < 1 || K > 32 || K >= n) return fail(GANNS_EINVAL, "K must be in [1, min(32, n-1)]");
+  if (max_iters < 0) return fail(GANNS_EINVAL, "max_iters < 0");
+  if (!aligned16(points)) return fail(GANNS_EINVAL, "points not 16-byte aligned");
+  for (int64_t v = 0; v < n; ++v)
+    for (int j = 0; j < K; ++j) {
+      const int32_t u = init_host[size_t(v) * K + j];
+      if (u < 0 || u >= n || u == v) return fail(GANNS_EINVAL, "init: ids must be in [0, n) and != row");
+      for (int i = 0; i < j; ++i)
+        if (init_host[size_t(v) * K + i] == u) return fail(GANNS_EINVAL, "init: repeated id in a row");
+    }
+  int rc = new_graph(n, d, K, metric, out);
+  if (rc) return rc;
+  int32_t* init_dev = nullptr;
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  cudaError_t e = cudaMalloc(&init_dev, sizeof(int32_t) * size_t(n) * K);
+  if (e == cudaSuccess)
+    e = cudaMemcpy(init_dev, init_host, sizeof(int32_t) * size_t(n) * K, cudaMemcpyHostToDevice);
+  if (e != cudaSuccess) {
+    cudaFree(init_dev);
+    ganns_graph_free(*out);
+    *out = nullptr;
+    return cuda_fail(e, "knn init upload");
+  }
+  int it = 0;
+  int64_t ch = 0;
+  rc = run_knn(points, n, d, metric == GANNS_COSINE ? GANNS_IP : metric, K, init_dev, max_iters,
+               (*out)->nbr, &it, &ch, s);
+  cudaFree(init_dev);
+  if (rc) {
+    ganns_graph_free(*out);
+    *out = nullptr;
+    return rc;
+  }
+  if (iters_out) *iters_out = it;
+  if (changed_last) *changed_last = ch;
+  return GANNS_OK;
+}
+
 int ganns_merge_topk(const int32_t* shard_ids, const float* shard_dists, int W, int64_t nq, int k,
                      int32_t* out_ids, float* out_dists, void* stream) {
   if (W < 1 || k < 1 || nq < 0) return fail(GANNS_EINVAL, "bad W / k / nq");

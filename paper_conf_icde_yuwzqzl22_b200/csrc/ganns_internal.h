@@ -100,6 +100,10 @@ int run_build(BuildArgs& a, cudaStream_t s);
 template <int NV4>
 int run_build_nv(BuildArgs& a, cudaStream_t s);
 
+int run_knn(const float* X, int64_t n, int d, int metric, int K, const int32_t* init_dev,
+            int max_iters, int32_t* out_ids, int* iters_out, int64_t* changed_last,
+            cudaStream_t s);
+
 cudaError_t launch_merge_topk(const int32_t* ids, const float* dists, int W, int64_t nq, int k,
                               int32_t* out_ids, float* out_dists, cudaStream_t s);
 cudaError_t launch_offset_ids(int32_t* ids, int64_t count, int64_t offset, cudaStream_t s);
