@@ -49,6 +49,8 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
     ap.add_argument("--json-out", default=None)
+    ap.add_argument("--shard-rows", type=int, default=0,
+                    help="C5 only: rows per shard (default: n / shards = 12.5M)")
     return ap.parse_args()
 
 
@@ -133,7 +135,7 @@ def make_workload(cfg, rank: int):
     return X, np.ascontiguousarray(Q)
 
 
-def ground_truth(torch, Xd, Qd, k, metric="l2"):
+def ground_truth(torch, Xd, Qd, k, metric="l2", with_dist=False):
     """Exact top-k by (dist, id) on the GPU in fp64 (bench-side measurement only).
     L2 on integer-grid data: every fp64 term is an exact integer, and the key
     dist * 2^21 + id (exact below 2^53) breaks ties by id.  IP / cosine (unit
@@ -141,7 +143,7 @@ def ground_truth(torch, Xd, Qd, k, metric="l2"):
     n = Xd.shape[0]
     Xd64, Qd64 = Xd.double(), Qd.double()
     best_k = best_i = None
-    shift = float(1 << 21)
+    shift = float(1 << max(21, int(n - 1).bit_length()))   # > every id: exact (dist, id) key
     for a in range(0, n, 65536):
         b = min(n, a + 65536)
         dot = Qd64 @ Xd64[a:b].T
@@ -158,6 +160,9 @@ def ground_truth(torch, Xd, Qd, k, metric="l2"):
             ck, ci = torch.cat([best_k, kk], 1), torch.cat([best_i, ki], 1)
             best_k, pos = torch.topk(ck, k, dim=1, largest=False, sorted=True)
             best_i = torch.gather(ci, 1, pos)
+    if with_dist:
+        dist = torch.floor(best_k / shift) if metric == "l2" else best_k
+        return best_i.int(), dist
     return best_i.int()
 
 
@@ -418,6 +423,136 @@ def run_ours(args):
         dist.destroy_process_group()
 
 
+def run_sharded(args):
+    """BASELINE configs[4] (DEEP100M-shaped, 100M x 96, 8 shards): every shard is an
+    independent NSW (Algorithm 2) over its rows; every query is searched on every
+    shard (K1), shard-local ids become global (id offset kernel), the per-shard
+    [nq, k] lists are all-gathered over NCCL and merged by K6 (ganns_merge_topk).
+    Rank r owns the shards s = r, r + N, ...; one step = the whole sharded search of
+    the 10K-query batch (strong scaling: the total work is fixed)."""
+    import torch
+    import torch.distributed as dist
+    import paper_conf_icde_yuwzqzl22_b200 as g
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    distributed = "RANK" in os.environ
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if distributed:
+        dist.init_process_group("nccl", device_id=dev)
+    cfg = syn.CONFIGS[args.config]
+    if args.shard_rows:
+        cfg = syn.with_size(cfg, n=args.shard_rows * cfg.shards)
+    k, W = cfg.k, cfg.shards
+    per = cfg.n // W
+    mine = [s for s in range(W) if s % world == rank]
+    Q = syn.queries(cfg)
+    Qd = torch.from_numpy(Q).to(dev)
+    nsub = min(1000, len(Q))                 # recall measured on a fixed query subset
+    shards, build_s, gt_parts = [], 0.0, []
+    for s in mine:
+        Xs = torch.from_numpy(syn.points(cfg, s * per, (s + 1) * per)).to(dev)
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        gr = g.build(Xs, metric=cfg.metric, degree=cfg.degree, l_build=args.l_build)
+        torch.cuda.synchronize()
+        build_s = max(build_s, time.perf_counter() - t0)
+        gi_s, gd_s = ground_truth(torch, Xs, Qd[:nsub], k, cfg.metric, with_dist=True)
+        gt_parts.append((gi_s.long() + s * per, gd_s))
+        shards.append((s, Xs, gr))
+    # exact top-k over all shards for the subset: each shard's exact top-k (fp64
+    # distances, exact on the integer grid) gathered and merged by (dist, global id)
+    cid = torch.cat([p for p, _ in gt_parts], 1)
+    cdd = torch.cat([d for _, d in gt_parts], 1)
+    if distributed:
+        ai = [torch.empty_like(cid) for _ in range(world)]
+        ad = [torch.empty_like(cdd) for _ in range(world)]
+        dist.all_gather(ai, cid)
+        dist.all_gather(ad, cdd)
+        cid, cdd = torch.cat(ai, 1), torch.cat(ad, 1)
+    key = cdd * float(1 << 27) + cid.double()
+    kk = torch.topk(key, k, dim=1, largest=False, sorted=True).values
+    gt = (kk - torch.floor(kk / float(1 << 27)) * float(1 << 27)).round().int()
+
+    def step(l, e, out_list=None):
+        ids_l, d_l = [], []
+        for s, Xs, gr in shards:
+            i, dd = g.search(gr, Xs, Qd, k, l, e=e)
+            g.offset_ids(i, s * per)
+            ids_l.append(i)
+            d_l.append(dd)
+        ids_loc, d_loc = torch.stack(ids_l), torch.stack(d_l)
+        if distributed:
+            gi = [torch.empty_like(ids_loc) for _ in range(world)]
+            gdd = [torch.empty_like(d_loc) for _ in range(world)]
+            dist.all_gather(gi, ids_loc)
+            dist.all_gather(gdd, d_loc)
+            ids_loc, d_loc = torch.cat(gi, 0), torch.cat(gdd, 0)
+        return g.merge_topk(ids_loc, d_loc)
+
+    chosen, sweep = None, []
+    for l in L_SWEEP:
+        ids, _ = step(l, l)
+        r = recall_at(ids[:nsub], gt)
+        sweep.append((l, round(r, 5)))
+        if r >= args.target:
+            chosen = l
+            break
+    l_star = chosen or L_SWEEP[-1]
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+    for _ in range(args.warmup):
+        step(l_star, l_star)
+    torch.cuda.synchronize()
+    if distributed:
+        dist.barrier()
+    launches0 = g.kernel_launches()
+    times = []
+    with ClockSampler(local) as clk:
+        for _ in range(args.steps):
+            flush.zero_()
+            torch.cuda.synchronize()
+            if distributed:
+                dist.barrier()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            ids, _ = step(l_star, l_star)
+            e1.record()
+            e1.synchronize()
+            times.append(e0.elapsed_time(e1) / 1e3)
+    launches = g.kernel_launches() - launches0
+    t = torch.tensor([sum(times)], dtype=torch.float64, device=dev)
+    if distributed:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    t_total = float(t.item())
+    rec = recall_at(ids[:nsub], gt)
+    qps = len(Q) * args.steps / t_total
+    line = {
+        "metric": "queries/sec at recall@10=0.95", "value": round(qps, 1), "unit": "queries/s",
+        "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": round(t_total / args.steps * 1e3, 3), "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+        "config": {"workload": f"{cfg.name}: DEEP-shaped {cfg.n}x{cfg.d} {cfg.metric}, {W} shards x "
+                               f"NSW degree {cfg.degree}, {len(Q)} queries, k={k}",
+                   "l": l_star, "e": l_star, "recall_at_10": round(rec, 5),
+                   "recall_subset": nsub, "l_sweep_recall": sweep,
+                   "shards_per_gpu": len(mine),
+                   "parallelism": f"base set sharded, {world} rank(s), NCCL all-gather + K6 merge",
+                   "l2": "flushed (256 MiB write) between timed steps"},
+        "build_seconds": round(build_s, 3), "build_note": "max over this run's shards (each built alone)",
+        "gpu_launches": int(launches), "clocks": clk.summary(),
+    }
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+        if args.json_out:
+            with open(args.json_out, "w") as f:
+                f.write(json.dumps(line) + "\n")
+    if distributed:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
 def cpu_baseline(index, X, Q, k, l, e, seconds):
     """The oracle's search (plain C, one pthread per host core) on a bounded sample
     of the same queries and graph.  Returns the cpu_baseline object."""
@@ -493,6 +628,8 @@ def main():
     args = parse()
     if args.impl == "reference":
         run_reference(args)
+    elif syn.CONFIGS[args.config].shards > 1:
+        run_sharded(args)
     else:
         run_ours(args)
 
