@@ -65,12 +65,6 @@ __device__ __forceinline__ unsigned lanemask_lt() {
   asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
   return m;
 }
-__device__ __forceinline__ float4 ldg_stream(const float4* p) {
-  float4 r;
-  asm("ld.global.nc.L1::no_allocate.v4.f32 {%0,%1,%2,%3}, [%4];"
-               : "=f"(r.x), "=f"(r.y), "=f"(r.z), "=f"(r.w) : "l"(p));
-  return r;
-}
 // Bulk L2 prefetch of one vector row (TMA unit, no registers held): issued for
 // every neighbour as soon as the adjacency row arrives, so the register-staged
 // loads of the bulk-distance passes find their lines in L2.
@@ -170,7 +164,25 @@ struct WarpSmem {
   uint32_t* sBM;
   uint32_t phase;   // parity of the next mbarrier phase to wait for
   int rounds;       // TMA rounds per exploration (1 or 2)
+  // CTA-shared stage pool (pool > 0): a warp holds a stage buffer only from its
+  // gather to the end of its distance math, so fewer buffers than warps suffice
+  int pool;
+  float4* pool_stage;       // pool buffers, pool_stride bytes apart
+  uint32_t pool_stride;
+  uint64_t* pool_mbar;      // one mbarrier per buffer
+  int* pool_owner;          // -1 = free
+  uint32_t* pool_phase;     // parity of each buffer's next phase
+  int held;                 // buffer held by this warp, -1 = none
 };
+// Per-CTA layout of the pooled search kernel: [pool stages][per-warp N/T/bitmap][pool meta]
+__host__ __device__ constexpr size_t pooled_warp_bytes(int l, int tpl) {
+  return (size_t(lpad32(l)) * 8 + size_t(tpl) * 32 * 8 + 16 + 128 + 15) & ~size_t(15);
+}
+__host__ __device__ constexpr size_t pooled_cta_bytes(int l, int tpl, int nv4, int d4, int rounds,
+                                                      int warps, int pool) {
+  return size_t(pool) * stage_bytes(nv4, d4, rounds) + size_t(warps) * pooled_warp_bytes(l, tpl) +
+         size_t(pool) * 16;
+}
 __device__ __forceinline__ WarpSmem carve_warp_smem(uint8_t* base, int l, int tpl, int nv4, int d4,
                                                    int rounds) {
   WarpSmem w;
@@ -181,7 +193,64 @@ __device__ __forceinline__ WarpSmem carve_warp_smem(uint8_t* base, int l, int tp
   w.mbar = w.sT + tpl * 32;
   w.sBM = reinterpret_cast<uint32_t*>(w.mbar + 2);
   w.phase = 0;
+  w.pool = 0;
+  w.held = -1;
   return w;
+}
+// pooled layout: warp w of `warps`; lane 0 of warp 0 initialises the pool
+__device__ __forceinline__ WarpSmem carve_pooled_smem(uint8_t* cta, int w, int warps, int pool, int l,
+                                                     int tpl, int nv4, int d4, int rounds) {
+  WarpSmem s;
+  s.rounds = rounds;
+  const size_t sb = stage_bytes(nv4, d4, rounds);
+  s.pool = pool;
+  s.pool_stage = reinterpret_cast<float4*>(cta);
+  s.pool_stride = uint32_t(sb);
+  uint8_t* wb = cta + size_t(pool) * sb + size_t(w) * pooled_warp_bytes(l, tpl);
+  s.sN = reinterpret_cast<uint64_t*>(wb);
+  s.sT = s.sN + lpad32(l);
+  s.mbar = nullptr;
+  s.sBM = reinterpret_cast<uint32_t*>(s.sT + tpl * 32 + 2);
+  uint8_t* meta = cta + size_t(pool) * sb + size_t(warps) * pooled_warp_bytes(l, tpl);
+  s.pool_mbar = reinterpret_cast<uint64_t*>(meta);
+  s.pool_owner = reinterpret_cast<int*>(s.pool_mbar + pool);
+  s.pool_phase = reinterpret_cast<uint32_t*>(s.pool_owner + pool);
+  s.stage = nullptr;
+  s.phase = 0;
+  s.held = -1;
+  return s;
+}
+// acquire a free pool buffer (lane 0 spins on the owner words), make it current
+__device__ __forceinline__ void stage_acquire(WarpSmem& ws, int lane) {
+  if (ws.pool == 0) return;
+  int b = -1;
+  if (lane == 0) {
+    const int me = int(threadIdx.x >> 5);
+    for (;;) {
+      for (int i = 0; i < ws.pool && b < 0; ++i)
+        if (atomicCAS(&ws.pool_owner[i], -1, me) == -1) b = i;
+      if (b >= 0) break;
+      __nanosleep(64);
+    }
+    __threadfence_block();
+  }
+  b = __shfl_sync(kFull, b, 0);
+  __syncwarp();
+  ws.held = b;
+  ws.stage = reinterpret_cast<float4*>(reinterpret_cast<char*>(ws.pool_stage) + size_t(b) * ws.pool_stride);
+  ws.mbar = ws.pool_mbar + b;
+  ws.phase = ws.pool_phase[b];
+}
+__device__ __forceinline__ void stage_release(WarpSmem& ws, int lane) {
+  if (ws.pool == 0) return;
+  __syncwarp();   // every lane's reads of the stage are done
+  if (lane == 0) {
+    ws.pool_phase[ws.held] = ws.phase;
+    __threadfence_block();
+    atomicExch(&ws.pool_owner[ws.held], -1);
+  }
+  __syncwarp();
+  ws.held = -1;
 }
 
 // Vector layout per dimension bucket (NV4 = template selector, see nv4_for):
@@ -251,6 +320,7 @@ __device__ __forceinline__ float tma_dot(const GraphView& g, const float4 (&qv)[
 #pragma unroll
   for (int f = 0; f < C; ++f) coff[f] = (FULL || sl + S * f < g.d4) ? sl + S * f : g.d4 - 1;
   float p[S];
+  stage_acquire(ws, lane);
 #pragma unroll
   for (int r = 0; r < ROUNDS; ++r) {
     // tile::gather4 (d % 8 == 0, so every group of 4 rows starts 128-B aligned):
@@ -310,6 +380,7 @@ __device__ __forceinline__ float tma_dot(const GraphView& g, const float4 (&qv)[
       p[r * PPR + gg] = hsum2(acc);
     }
   }
+  stage_release(ws, lane);
 #pragma unroll
   for (int half = S / 2; half >= 1; half >>= 1) {
     const bool up = lane & half;
@@ -334,6 +405,7 @@ __device__ __forceinline__ float wide_dot(const GraphView& g, const float4 (&qv)
   constexpr int R = kWideStageRows;   // 8 rows per round, 4 rounds
   const uint32_t rowbytes = uint32_t(g.d4) * 16u;
   float dres = 0.f;
+  stage_acquire(ws, lane);
 #pragma unroll 1
   for (int r = 0; r < 32 / R; ++r) {
     const bool mine = u_mine >= 0 && (lane / R) == r;
@@ -378,6 +450,7 @@ __device__ __forceinline__ float wide_dot(const GraphView& g, const float4 (&qv)
     const float got = __shfl_sync(kFull, p[0], (lane % R) << 2);
     if (lane / R == r) dres = got;
   }
+  stage_release(ws, lane);
   return dres;
 }
 

@@ -19,7 +19,14 @@ struct ganns_graph {
 namespace ganns {
 
 constexpr int kWarpsPerBlock = 4;   // warps per CTA of the small helper kernels
-constexpr int kSearchWarps = 2;     // warps (= concurrent queries) per CTA of the search kernel
+#ifndef GANNS_SEARCH_WARPS
+#define GANNS_SEARCH_WARPS 2
+#endif
+#ifndef GANNS_SEARCH_POOL
+#define GANNS_SEARCH_POOL 0
+#endif
+constexpr int kSearchWarps = GANNS_SEARCH_WARPS;   // warps (= concurrent queries) per CTA
+constexpr int kSearchPool = GANNS_SEARCH_POOL;     // shared stage buffers per CTA (0: one per warp)
 #ifndef GANNS_MIN_BLOCKS
 #define GANNS_MIN_BLOCKS 12
 #endif

@@ -23,11 +23,22 @@ search_kernel(GraphView g, const float* __restrict__ Q, int64_t nq, int k, int l
   g.tmap = &tmap;
   extern __shared__ __align__(128) uint8_t smem[];
   const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  WarpSmem ws = carve_warp_smem(
-      smem + size_t(w) * warp_smem_bytes(l, TPL, NV4, g.d4, kSearchStageRounds), l, TPL, NV4, g.d4,
-      kSearchStageRounds);
-  if (lane == 0) mbar_init(ws.mbar, 1);
-  __syncwarp();
+  WarpSmem ws;
+  if constexpr (kSearchPool > 0) {
+    ws = carve_pooled_smem(smem, w, kSearchWarps, kSearchPool, l, TPL, NV4, g.d4,
+                           kSearchStageRounds);
+    if (w == 0 && lane < kSearchPool) {
+      mbar_init(ws.pool_mbar + lane, 1);
+      ws.pool_owner[lane] = -1;
+      ws.pool_phase[lane] = 0;
+    }
+    __syncthreads();
+  } else {
+    ws = carve_warp_smem(smem + size_t(w) * warp_smem_bytes(l, TPL, NV4, g.d4, kSearchStageRounds),
+                         l, TPL, NV4, g.d4, kSearchStageRounds);
+    if (lane == 0) mbar_init(ws.mbar, 1);
+    __syncwarp();
+  }
   uint64_t* sN = ws.sN;
   for (;;) {
   int32_t qt = 0;
@@ -57,8 +68,10 @@ search_kernel(GraphView g, const float* __restrict__ Q, int64_t nq, int k, int l
 template <int NV4, int TPL, bool L2>
 static cudaError_t launch_t(const SearchLaunch& a, cudaStream_t s) {
   auto kern = search_kernel<NV4, TPL, L2>;
-  size_t smem =
-      size_t(kSearchWarps) * warp_smem_bytes(a.l, TPL, NV4, a.d / 4, kSearchStageRounds);
+  size_t smem = kSearchPool > 0
+                    ? pooled_cta_bytes(a.l, TPL, NV4, a.d / 4, kSearchStageRounds, kSearchWarps,
+                                       kSearchPool)
+                    : size_t(kSearchWarps) * warp_smem_bytes(a.l, TPL, NV4, a.d / 4, kSearchStageRounds);
   static bool attr_done = false;   // per instantiation
   if (!attr_done) {
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
