@@ -406,6 +406,10 @@ def run_ours(args):
         "gpu_launches": int(launches),
         "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak,
                      "unit": "GB/s", "frac": round(achieved / peak, 4), "traffic": traffic,
+                     # measured DRAM bytes (ncu, cold L2) over the live launch time: the
+                     # algorithmic figure above counts L2 hits as well, so it can exceed 1
+                     "traffic_frac": (round(traffic / kernel_s / 1e9 / peak, 4)
+                                      if traffic else None),
                      "peak_kind": peak_kind, "alg_bytes_per_launch": alg_bytes,
                      "kernel": f"ganns::search_kernel (d={cfg.d}, d_max={cfg.degree}, {cfg.metric})"},
         "clocks": clk.summary(),
@@ -476,10 +480,15 @@ def run_sharded(args):
     kk = torch.topk(key, k, dim=1, largest=False, sorted=True).values
     gt = (kk - torch.floor(kk / float(1 << 27)) * float(1 << 27)).round().int()
 
-    def step(l, e, out_list=None):
+    def step(l, e, ev=None, Qin=None):
         ids_l, d_l = [], []
         for s, Xs, gr in shards:
-            i, dd = g.search(gr, Xs, Qd, k, l, e=e)
+            if ev is not None:
+                ev.append((torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)))
+                ev[-1][0].record()
+            i, dd = g.search(gr, Xs, Qd if Qin is None else Qin, k, l, e=e)
+            if ev is not None:
+                ev[-1][1].record()
             g.offset_ids(i, s * per)
             ids_l.append(i)
             d_l.append(dd)
@@ -508,7 +517,7 @@ def run_sharded(args):
     if distributed:
         dist.barrier()
     launches0 = g.kernel_launches()
-    times = []
+    times, sev = [], []
     with ClockSampler(local) as clk:
         for _ in range(args.steps):
             flush.zero_()
@@ -517,7 +526,7 @@ def run_sharded(args):
                 dist.barrier()
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record()
-            ids, _ = step(l_star, l_star)
+            ids, _ = step(l_star, l_star, ev=sev)
             e1.record()
             e1.synchronize()
             times.append(e0.elapsed_time(e1) / 1e3)
@@ -528,6 +537,39 @@ def run_sharded(args):
     t_total = float(t.item())
     rec = recall_at(ids[:nsub], gt)
     qps = len(Q) * args.steps / t_total
+    # roofline of K1 on the shards (untimed stats pass: the kernel's own counters)
+    search_s = sum(a.elapsed_time(b) for a, b in sev) / 1e3 / max(1, len(sev))
+    alg = 0
+    for s, Xs, gr in shards:
+        _, _, st = g.search(gr, Xs, Qd, k, l_star, e=l_star, stats=True)
+        st = st.long()
+        alg += int((4 * cfg.d + 4 * cfg.degree * st[:, 0] + 4 * cfg.d * st[:, 1]).sum()) + 8 * k * len(Q)
+    alg_per_launch = alg // max(1, len(shards))
+    peak, peak_kind = peaks()
+    achieved = alg_per_launch / search_s / 1e9
+    # end to end: queries from pinned host memory, results back to pinned host
+    # memory, inside the timed region (the all-gather and merge included)
+    Qh = torch.from_numpy(Q).pin_memory()
+    Qin = torch.empty_like(Qd)
+    hid = torch.empty((len(Q), k), dtype=torch.int32).pin_memory()
+    hdd = torch.empty((len(Q), k), dtype=torch.float32).pin_memory()
+    e2e = []
+    for it in range(args.warmup + args.steps):
+        torch.cuda.synchronize()
+        if distributed:
+            dist.barrier()
+        t0 = time.perf_counter()
+        Qin.copy_(Qh, non_blocking=True)
+        i_, d_ = step(l_star, l_star, Qin=Qin)
+        hid.copy_(i_, non_blocking=True)
+        hdd.copy_(d_, non_blocking=True)
+        torch.cuda.current_stream().synchronize()
+        if it >= args.warmup:
+            e2e.append(time.perf_counter() - t0)
+    te = torch.tensor([sum(e2e)], dtype=torch.float64, device=dev)
+    if distributed:
+        dist.all_reduce(te, op=dist.ReduceOp.MAX)
+    e2e_qps = len(Q) * args.steps / float(te.item())
     line = {
         "metric": "queries/sec at recall@10=0.95", "value": round(qps, 1), "unit": "queries/s",
         "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
@@ -542,7 +584,17 @@ def run_sharded(args):
                    "l2": "flushed (256 MiB write) between timed steps"},
         "build_seconds": round(build_s, 3), "build_note": "max over this run's shards (each built alone)",
         "gpu_launches": int(launches), "clocks": clk.summary(),
+        "e2e": {"value": round(e2e_qps, 1), "unit": "queries/s",
+                "h2d_bytes_per_step": int(Q.nbytes), "d2h_bytes_per_step": int(len(Q) * k * 8)},
+        "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
+                     "frac": round(achieved / peak, 4), "traffic": None, "peak_kind": peak_kind,
+                     "alg_bytes_per_launch": alg_per_launch,
+                     "kernel": f"ganns::search_kernel on one {per}-row shard (d={cfg.d}, "
+                               f"d_max={cfg.degree}, {cfg.metric}); mean over the shard launches"},
     }
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        line["cpu_baseline"] = sharded_cpu_baseline(torch, g, shards, per, Q, k, l_star,
+                                                    args.cpu_seconds, cfg.metric)
     if rank == 0:
         print(json.dumps(line), flush=True)
         if args.json_out:
@@ -551,6 +603,36 @@ def run_sharded(args):
     if distributed:
         dist.barrier()
         dist.destroy_process_group()
+
+
+def sharded_cpu_baseline(torch, g, shards, per, Q, k, l, seconds, metric):
+    """The oracle's sharded search on a bounded query sample: every shard searched by
+    the oracle (plain C, one pthread per host core, same graph and l), then the
+    oracle's merge by (dist, global id).  Host copies of the shards (not timed)."""
+    import oracle
+    cores = oracle.ncores()
+    m = 0
+    for s, Xs, gr in shards[:1]:   # calibrate the sample on the first shard
+        Xh, A = Xs.cpu().numpy(), gr.adjacency()
+        t0 = time.perf_counter()
+        oracle.search(A, Xh, Q[:32], k, l, e=l, metric=metric, threads=cores)
+        dt = time.perf_counter() - t0
+        m = int(min(len(Q), max(32, 32 * seconds / max(dt * len(shards), 1e-3))))
+        del Xh, A
+    tot, parts = 0.0, []
+    for s, Xs, gr in shards:
+        Xh, A = Xs.cpu().numpy(), gr.adjacency()
+        t0 = time.perf_counter()
+        ids, dd = oracle.search(A, Xh, Q[:m], k, l, e=l, metric=metric, threads=cores)
+        tot += time.perf_counter() - t0
+        parts.append((np.where(ids >= 0, ids + s * per, -1).astype(np.int32), dd))
+        del Xh, A
+    t0 = time.perf_counter()
+    oracle.merge_topk(np.stack([p[0] for p in parts]), np.stack([p[1] for p in parts]))
+    tot += time.perf_counter() - t0
+    return {"value": round(m / tot, 1), "unit": "queries/s", "cores": cores, "kind": "oracle",
+            "sample": f"first {m} of the {len(Q)} queries on all {len(shards)} shards "
+                      f"(same graphs, l={l}) + merge, {tot:.1f} s"}
 
 
 def cpu_baseline(index, X, Q, k, l, e, seconds):

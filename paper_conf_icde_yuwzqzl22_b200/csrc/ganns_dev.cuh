@@ -127,6 +127,11 @@ struct GraphView {
   int d_max;
   int d4;               // d / 4
   int metric;           // 0 L2, 1 IP, 2 COSINE
+  // L2 residency hint (0 = none): vector rows of vertices < hot are fetched with
+  // an evict_last policy (the early-inserted hubs every search passes through),
+  // the others with evict_first when cold_first is set
+  int32_t hot = 0;
+  int32_t cold_first = 0;
 };
 
 // Per-search counters (kept in registers, identical to the oracle's stats[0,1,3]).
@@ -146,15 +151,22 @@ constexpr int kWideStageRows = 8;   // d > 256: rows per TMA round (4 rounds per
 #ifndef GANNS_SEARCH_ROUNDS
 #define GANNS_SEARCH_ROUNDS 2
 #endif
+#ifndef GANNS_PREFETCH_R2
+#define GANNS_PREFETCH_R2 0
+#endif
 constexpr int kSearchStageRounds = GANNS_SEARCH_ROUNDS;
 constexpr int kBuildStageRounds = 1;
-__host__ __device__ constexpr size_t stage_bytes(int nv4, int d4, int rounds) {
-  return uses_tma(nv4) ? size_t(32 / rounds) * d4 * 16 : size_t(kWideStageRows) * d4 * 16;
+// wrows: rows per TMA round of the wide (d > 256) form, 1..kWideStageRows (the
+// search launcher lowers it so that a small batch fits one wave of warps)
+__host__ __device__ constexpr size_t stage_bytes(int nv4, int d4, int rounds,
+                                                 int wrows = kWideStageRows) {
+  return uses_tma(nv4) ? size_t(32 / rounds) * d4 * 16 : size_t(wrows) * d4 * 16;
 }
-__host__ __device__ constexpr size_t warp_smem_bytes(int l, int tpl, int nv4, int d4, int rounds) {
+__host__ __device__ constexpr size_t warp_smem_bytes(int l, int tpl, int nv4, int d4, int rounds,
+                                                     int wrows = kWideStageRows) {
   // rounded to 128 B: the stage (first) must be 128-B aligned for tensor TMA
-  return (stage_bytes(nv4, d4, rounds) + size_t(lpad32(l)) * 8 + size_t(tpl) * 32 * 8 + 16 + 128 +
-          127) & ~size_t(127);
+  return (stage_bytes(nv4, d4, rounds, wrows) + size_t(lpad32(l)) * 8 + size_t(tpl) * 32 * 8 + 16 +
+          128 + 127) & ~size_t(127);
 }
 struct WarpSmem {
   float4* stage;
@@ -164,6 +176,7 @@ struct WarpSmem {
   uint32_t* sBM;
   uint32_t phase;   // parity of the next mbarrier phase to wait for
   int rounds;       // TMA rounds per exploration (1 or 2)
+  int wrows;        // wide form: rows per TMA round (1..kWideStageRows)
   // CTA-shared stage pool (pool > 0): a warp holds a stage buffer only from its
   // gather to the end of its distance math, so fewer buffers than warps suffice
   int pool;
@@ -184,11 +197,12 @@ __host__ __device__ constexpr size_t pooled_cta_bytes(int l, int tpl, int nv4, i
          size_t(pool) * 16;
 }
 __device__ __forceinline__ WarpSmem carve_warp_smem(uint8_t* base, int l, int tpl, int nv4, int d4,
-                                                   int rounds) {
+                                                   int rounds, int wrows = kWideStageRows) {
   WarpSmem w;
   w.rounds = rounds;
+  w.wrows = wrows;
   w.stage = reinterpret_cast<float4*>(base);
-  w.sN = reinterpret_cast<uint64_t*>(base + stage_bytes(nv4, d4, rounds));
+  w.sN = reinterpret_cast<uint64_t*>(base + stage_bytes(nv4, d4, rounds, wrows));
   w.sT = w.sN + lpad32(l);
   w.mbar = w.sT + tpl * 32;
   w.sBM = reinterpret_cast<uint32_t*>(w.mbar + 2);
@@ -202,6 +216,7 @@ __device__ __forceinline__ WarpSmem carve_pooled_smem(uint8_t* cta, int w, int w
                                                      int tpl, int nv4, int d4, int rounds) {
   WarpSmem s;
   s.rounds = rounds;
+  s.wrows = kWideStageRows;
   const size_t sb = stage_bytes(nv4, d4, rounds);
   s.pool = pool;
   s.pool_stage = reinterpret_cast<float4*>(cta);
@@ -320,6 +335,14 @@ __device__ __forceinline__ float tma_dot(const GraphView& g, const float4 (&qv)[
 #pragma unroll
   for (int f = 0; f < C; ++f) coff[f] = (FULL || sl + S * f < g.d4) ? sl + S * f : g.d4 - 1;
   float p[S];
+#if GANNS_PREFETCH_R2
+  // rows of the later rounds start towards L2 now (no extra traffic: they are read
+  // by this exploration's next TMA round)
+  if constexpr (ROUNDS > 1)
+    if (u_mine >= 0 && my_round > 0)
+      prefetch_row_l2(reinterpret_cast<const char*>(g.X) + uint64_t(uint32_t(u_mine)) * rowbytes,
+                      rowbytes);
+#endif
   stage_acquire(ws, lane);
 #pragma unroll
   for (int r = 0; r < ROUNDS; ++r) {
@@ -354,7 +377,23 @@ __device__ __forceinline__ float tma_dot(const GraphView& g, const float4 (&qv)[
       __syncwarp();
       char* dst = reinterpret_cast<char*>(ws.stage) + size_t(my_slot) * rowbytes;
       if (issuer) {
-        if (g4)
+        if (g4 && g.hot > 0) {
+          // absent rows carry 0x7fffffff: never hot
+          const bool hot4 = uo < g.hot || u1 < g.hot || u2 < g.hot || u3 < g.hot;
+          uint64_t pol;
+          if (hot4)
+            asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
+          else if (g.cold_first)
+            asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+          else
+            asm("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(pol));
+          asm volatile(
+              "cp.async.bulk.tensor.2d.shared::cta.global.tile::gather4.mbarrier::complete_tx::bytes"
+              ".L2::cache_hint [%0], [%1, {%2, %3, %4, %5, %6}], [%7], %8;" ::"r"(smem_u32(dst)),
+              "l"(g.tmap), "r"(0), "r"(uo), "r"(u1), "r"(u2), "r"(u3), "r"(smem_u32(ws.mbar)),
+              "l"(pol)
+              : "memory");
+        } else if (g4)
           asm volatile(
               "cp.async.bulk.tensor.2d.shared::cta.global.tile::gather4.mbarrier::complete_tx::bytes"
               " [%0], [%1, {%2, %3, %4, %5, %6}], [%7];" ::"r"(smem_u32(dst)),
@@ -394,21 +433,24 @@ __device__ __forceinline__ float tma_dot(const GraphView& g, const float4 (&qv)[
   return p[0];
 }
 
-// Whole-warp form (S = 32, d > 256): rows are staged kWideStageRows at a time by
-// 1-D TMA bulk copies (one per row, issued by the lane owning the neighbour);
-// each lane reads float4 columns lane + 32f of every staged row from shared
-// memory; per round a transposing butterfly over the top 3 lane bits and a plain
-// reduction over the rest leave lane j with row j's total.
+// Whole-warp form (S = 32, d > 256): rows are staged R = ws.wrows (<= 8) at a
+// time by 1-D TMA bulk copies (one per row, issued by the lane owning the
+// neighbour), ceil(32 / R) rounds; each lane reads float4 columns lane + 32f of
+// every staged row from shared memory; per round a transposing butterfly over
+// the top 3 lane bits (8 slots; slots >= R add 0) and a plain reduction over the
+// rest leave lane j with row j's total.
 template <int C, bool L2, bool FULL>
 __device__ __forceinline__ float wide_dot(const GraphView& g, const float4 (&qv)[C],
                                           int32_t u_mine, int lane, WarpSmem& ws) {
-  constexpr int R = kWideStageRows;   // 8 rows per round, 4 rounds
+  constexpr int RM = kWideStageRows;   // butterfly width
+  const int R = ws.wrows;
+  const int my_round = lane / R, my_slot = lane - my_round * R;
   const uint32_t rowbytes = uint32_t(g.d4) * 16u;
   float dres = 0.f;
   stage_acquire(ws, lane);
 #pragma unroll 1
-  for (int r = 0; r < 32 / R; ++r) {
-    const bool mine = u_mine >= 0 && (lane / R) == r;
+  for (int r = 0; r * R < 32; ++r) {
+    const bool mine = u_mine >= 0 && my_round == r;
     const unsigned vm = __ballot_sync(kFull, mine);
     if (vm) {
       __syncwarp();
@@ -416,26 +458,28 @@ __device__ __forceinline__ float wide_dot(const GraphView& g, const float4 (&qv)
       if (lane == 0) mbar_arrive_expect_tx(ws.mbar, uint32_t(__popc(vm)) * rowbytes);
       __syncwarp();
       if (mine)
-        tma_row(reinterpret_cast<char*>(ws.stage) + size_t(lane % R) * rowbytes,
+        tma_row(reinterpret_cast<char*>(ws.stage) + size_t(my_slot) * rowbytes,
                 reinterpret_cast<const char*>(g.X) + uint64_t(uint32_t(u_mine)) * rowbytes,
                 rowbytes, ws.mbar);
       mbar_wait(ws.mbar, ws.phase);
       ws.phase ^= 1u;
     }
-    float p[R];
+    float p[RM];
 #pragma unroll
-    for (int i = 0; i < R; ++i) {
-      const float4* rp = ws.stage + size_t(i) * g.d4;
+    for (int i = 0; i < RM; ++i) {
       uint64_t acc = 0;
+      if (i < R) {
+        const float4* rp = ws.stage + size_t(i) * g.d4;
 #pragma unroll
-      for (int f = 0; f < C; ++f)
-        if (FULL || lane + 32 * f < g.d4) acc = accum4<L2>(acc, qv[f], rp[lane + 32 * f]);
+        for (int f = 0; f < C; ++f)
+          if (FULL || lane + 32 * f < g.d4) acc = accum4<L2>(acc, qv[f], rp[lane + 32 * f]);
+      }
       p[i] = hsum2(acc);
     }
-    // transposing butterfly over lane bits 4,3,2 (8 rows), then bits 1,0
+    // transposing butterfly over lane bits 4,3,2 (8 slots), then bits 1,0
 #pragma unroll
     for (int st = 0; st < 3; ++st) {
-      const int half = R >> (st + 1), off = 16 >> st;
+      const int half = RM >> (st + 1), off = 16 >> st;
       const bool up = lane & off;
 #pragma unroll
       for (int i = 0; i < half; ++i) {
@@ -446,9 +490,9 @@ __device__ __forceinline__ float wide_dot(const GraphView& g, const float4 (&qv)
     }
     p[0] += __shfl_xor_sync(kFull, p[0], 2);
     p[0] += __shfl_xor_sync(kFull, p[0], 1);
-    // lane L holds the total of row (L >> 2) of this round
-    const float got = __shfl_sync(kFull, p[0], (lane % R) << 2);
-    if (lane / R == r) dres = got;
+    // lane L holds the total of slot (L >> 2) of this round
+    const float got = __shfl_sync(kFull, p[0], (my_slot & (RM - 1)) << 2);
+    if (my_round == r) dres = got;
   }
   stage_release(ws, lane);
   return dres;
@@ -484,45 +528,69 @@ __device__ __forceinline__ float group_distances(const GraphView& g,
 }
 
 
+// Bulk-distance policy of one warp (the default): the query slice lives in this
+// warp's registers and the warp computes all distances of an exploration itself.
+template <int NV4, bool L2>
+struct WarpDist {
+  static constexpr int S = VecLayout<NV4>::S, C = VecLayout<NV4>::C;
+  float4 qv[C];
+  float cbase, qinv;
+  // query slice in registers (P:197-199, P:224): lane owns float4 columns
+  // lane%S + S*f (every S-lane segment holds a full copy of q)
+  __device__ __forceinline__ void load(const GraphView& g, const float* __restrict__ qrow, int lane) {
+    const float4* q4 = reinterpret_cast<const float4*>(qrow);
+#pragma unroll
+    for (int f = 0; f < C; ++f) {
+      int i4 = (lane & (S - 1)) + S * f;
+      qv[f] = i4 < g.d4 ? q4[i4] : make_float4(0.f, 0.f, 0.f, 0.f);
+    }
+    cbase = 0.f;
+    qinv = 1.f;
+    if (!L2 && g.metric == 2) {
+      float s = 0.f;
+#pragma unroll
+      for (int f = 0; f < C; ++f)
+        s += qv[f].x * qv[f].x + qv[f].y * qv[f].y + qv[f].z * qv[f].z + qv[f].w * qv[f].w;
+#pragma unroll
+      for (int off = S / 2; off >= 1; off >>= 1) s += __shfl_xor_sync(kFull, s, off);
+      cbase = 1.f;
+      qinv = 1.f / sqrtf(s);
+    }
+  }
+  // wide rows are staged in several rounds: warm the later rounds' rows in L2 as
+  // soon as the adjacency row is known
+  __device__ __forceinline__ void explore_hint(const GraphView& g, int32_t u_mine, int lane,
+                                               const WarpSmem& ws) {
+    if constexpr (!uses_tma(NV4))
+      if (u_mine >= 0 && lane >= ws.wrows)
+        prefetch_row_l2(g.X + size_t(u_mine) * (g.d4 * 4), uint32_t(g.d4) * 16u);
+  }
+  __device__ __forceinline__ float operator()(const GraphView& g, int32_t u_mine, int lane,
+                                              WarpSmem& ws) {
+    return group_distances<NV4, L2>(g, qv, u_mine, cbase, qinv, lane, ws);
+  }
+};
+
 // The GANNS search of one query by one warp.  On return sN[0..cnt) holds N
 // (ascending, explored flags set); returns cnt.  COHERENT: read the graph with
-// coherent loads (the build modifies it inside the same kernel).
-template <int NV4, int TPL, bool L2, bool COHERENT>
-__device__ int warp_search(const GraphView& g, const float* __restrict__ qrow, int32_t entry,
-                           int l, int e, WarpSmem& ws, SearchStats& st) {
+// coherent loads (the build modifies it inside the same kernel).  DIST computes
+// the bulk distances of one exploration (WarpDist: this warp alone; GroupDist:
+// this warp and its helper warps, search_group.cu).
+template <class DIST, int TPL, bool COHERENT>
+__device__ int warp_search_with(const GraphView& g, DIST& dist, int32_t entry, int l, int e,
+                                WarpSmem& ws, SearchStats& st) {
   const int lane = threadIdx.x & 31;
   uint64_t* sN = ws.sN;
   uint64_t* sT = ws.sT;
   uint32_t* sBM = ws.sBM;
   const int lp = lpad32(l);
   const int nwords = lp >> 5;
-  // query slice in registers (P:197-199, P:224): lane owns float4 columns
-  // lane%S + S*f (every S-lane segment holds a full copy of q)
-  constexpr int S = VecLayout<NV4>::S, C = VecLayout<NV4>::C;
-  float4 qv[C];
-  const float4* q4 = reinterpret_cast<const float4*>(qrow);
-#pragma unroll
-  for (int f = 0; f < C; ++f) {
-    int i4 = (lane & (S - 1)) + S * f;
-    qv[f] = i4 < g.d4 ? q4[i4] : make_float4(0.f, 0.f, 0.f, 0.f);
-  }
-  float cbase = 0.f, qinv = 1.f;
-  if (!L2 && g.metric == 2) {
-    float s = 0.f;
-#pragma unroll
-    for (int f = 0; f < C; ++f)
-      s += qv[f].x * qv[f].x + qv[f].y * qv[f].y + qv[f].z * qv[f].z + qv[f].w * qv[f].w;
-#pragma unroll
-    for (int off = S / 2; off >= 1; off >>= 1) s += __shfl_xor_sync(kFull, s, off);
-    cbase = 1.f;
-    qinv = 1.f / sqrtf(s);
-  }
   // init: N = [(delta(q, entry), entry, unexplored)]
   for (int i = lane; i < lp; i += 32) sN[i] = kKeyInf;
   if (lane < nwords) sBM[lane] = 0u;
   {
     int32_t u = lane == 0 ? entry : -1;
-    float dd = group_distances<NV4, L2>(g, qv, u, cbase, qinv, lane, ws);
+    float dd = dist(g, u, lane, ws);
     if (lane == 0) sN[0] = mkkey(dd, entry);
   }
   __syncwarp();
@@ -576,18 +644,12 @@ __device__ int warp_search(const GraphView& g, const float* __restrict__ qrow, i
     }
     spec_v = w;
     // (3) bulk distance computation
-    if constexpr (!uses_tma(NV4)) {
-      // wide rows are staged in 4 rounds: warm all of them in L2 at once so the
-      // later rounds find their lines close
 #pragma unroll
-      for (int t = 0; t < TPL; ++t)
-        if (u[t] >= 0 && (lane / kWideStageRows) != 0)
-          prefetch_row_l2(g.X + size_t(u[t]) * (g.d4 * 4), uint32_t(g.d4) * 16u);
-    }
+    for (int t = 0; t < TPL; ++t) dist.explore_hint(g, u[t], lane, ws);
     uint64_t key[TPL];
 #pragma unroll
     for (int t = 0; t < TPL; ++t) {
-      float dd = group_distances<NV4, L2>(g, qv, u[t], cbase, qinv, lane, ws);
+      float dd = dist(g, u[t], lane, ws);
       key[t] = u[t] >= 0 ? mkkey(dd, u[t]) : kKeyInf;
       st.comps += __popc(__ballot_sync(kFull, u[t] >= 0));
     }
@@ -695,6 +757,15 @@ __device__ int warp_search(const GraphView& g, const float* __restrict__ qrow, i
     __syncwarp();
   }
   return cnt;
+}
+
+template <int NV4, int TPL, bool L2, bool COHERENT>
+__device__ __forceinline__ int warp_search(const GraphView& g, const float* __restrict__ qrow,
+                                           int32_t entry, int l, int e, WarpSmem& ws,
+                                           SearchStats& st) {
+  WarpDist<NV4, L2> dist;
+  dist.load(g, qrow, threadIdx.x & 31);
+  return warp_search_with<WarpDist<NV4, L2>, TPL, COHERENT>(g, dist, entry, l, e, ws, st);
 }
 
 // ---------------------------------------------------------------- HNSW

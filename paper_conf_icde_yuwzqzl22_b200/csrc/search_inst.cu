@@ -3,6 +3,7 @@
 // instances build in parallel.  See ganns_dev.cuh for the algorithm.
 #include "ganns_dev.cuh"
 #include "ganns_internal.h"
+#include "search_group.cuh"
 
 #include <cstdlib>
 
@@ -19,7 +20,8 @@ __global__ void __launch_bounds__(kSearchWarps * 32, kMinBlocksPerSM)
 search_kernel(GraphView g, const float* __restrict__ Q, int64_t nq, int k, int l, int e,
               int32_t entry, int32_t* __restrict__ out_ids, float* __restrict__ out_dists,
               uint32_t* __restrict__ stats, int32_t* __restrict__ ticket,
-              const int32_t* __restrict__ entries, const __grid_constant__ CUtensorMap tmap) {
+              const int32_t* __restrict__ entries, int wrows,
+              const __grid_constant__ CUtensorMap tmap) {
   g.tmap = &tmap;
   extern __shared__ __align__(128) uint8_t smem[];
   const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -34,8 +36,9 @@ search_kernel(GraphView g, const float* __restrict__ Q, int64_t nq, int k, int l
     }
     __syncthreads();
   } else {
-    ws = carve_warp_smem(smem + size_t(w) * warp_smem_bytes(l, TPL, NV4, g.d4, kSearchStageRounds),
-                         l, TPL, NV4, g.d4, kSearchStageRounds);
+    ws = carve_warp_smem(
+        smem + size_t(w) * warp_smem_bytes(l, TPL, NV4, g.d4, kSearchStageRounds, wrows), l, TPL,
+        NV4, g.d4, kSearchStageRounds, wrows);
     if (lane == 0) mbar_init(ws.mbar, 1);
     __syncwarp();
   }
@@ -65,13 +68,33 @@ search_kernel(GraphView g, const float* __restrict__ Q, int64_t nq, int k, int l
   }
 }
 
+// Rows per TMA round of the wide form (d > 256): the largest R <= 8 whose
+// resident warps hold the whole batch in one wave (a second, nearly empty wave
+// would cost a full query latency); R = 8 when no R >= 4 fits.  GANNS_WIDE_ROWS
+// overrides (developer knob).
+template <int NV4, int TPL, bool L2>
+static int pick_wide_rows(const SearchLaunch& a, int sms) {
+  if (uses_tma(NV4)) return kWideStageRows;
+  static const int forced = [] {
+    const char* e = std::getenv("GANNS_WIDE_ROWS");
+    return e ? std::atoi(e) : 0;
+  }();
+  if (forced >= 1 && forced <= kWideStageRows) return forced;
+  for (int r = kWideStageRows; r >= 4; --r) {
+    int per_sm = 0;
+    const size_t smem = size_t(kSearchWarps) * warp_smem_bytes(a.l, TPL, NV4, a.d / 4,
+                                                               kSearchStageRounds, r);
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, search_kernel<NV4, TPL, L2>,
+                                                      kSearchWarps * 32, smem) != cudaSuccess)
+      return kWideStageRows;
+    if (int64_t(per_sm) * sms * kSearchWarps >= a.nq) return r;
+  }
+  return kWideStageRows;
+}
+
 template <int NV4, int TPL, bool L2>
 static cudaError_t launch_t(const SearchLaunch& a, cudaStream_t s) {
   auto kern = search_kernel<NV4, TPL, L2>;
-  size_t smem = kSearchPool > 0
-                    ? pooled_cta_bytes(a.l, TPL, NV4, a.d / 4, kSearchStageRounds, kSearchWarps,
-                                       kSearchPool)
-                    : size_t(kSearchWarps) * warp_smem_bytes(a.l, TPL, NV4, a.d / 4, kSearchStageRounds);
   static bool attr_done = false;   // per instantiation
   if (!attr_done) {
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -81,6 +104,15 @@ static cudaError_t launch_t(const SearchLaunch& a, cudaStream_t s) {
     if (e != cudaSuccess) return e;
     attr_done = true;
   }
+  int dev = 0, sms = 0, per_sm = 0;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  const int wrows = kSearchPool > 0 ? kWideStageRows : pick_wide_rows<NV4, TPL, L2>(a, sms);
+  size_t smem = kSearchPool > 0
+                    ? pooled_cta_bytes(a.l, TPL, NV4, a.d / 4, kSearchStageRounds, kSearchWarps,
+                                       kSearchPool)
+                    : size_t(kSearchWarps) *
+                          warp_smem_bytes(a.l, TPL, NV4, a.d / 4, kSearchStageRounds, wrows);
   if (smem > 227 * 1024) return cudaErrorInvalidValue;
   {
     // developer knob (occupancy experiments): extra shared memory per CTA
@@ -91,12 +123,22 @@ static cudaError_t launch_t(const SearchLaunch& a, cudaStream_t s) {
     smem += size_t(pad);
   }
   GraphView g{a.nbr, a.X, nullptr, a.n, a.d_max, a.d / 4, a.metric};
+  {
+    // developer knobs (L2 residency experiments): GANNS_L2_HOT_ROWS, GANNS_L2_COLD_FIRST
+    static const int hot = [] {
+      const char* e = std::getenv("GANNS_L2_HOT_ROWS");
+      return e ? std::atoi(e) : 0;
+    }();
+    static const int cold_first = [] {
+      const char* e = std::getenv("GANNS_L2_COLD_FIRST");
+      return e ? std::atoi(e) : 0;
+    }();
+    g.hot = hot;
+    g.cold_first = cold_first;
+  }
   CUtensorMap tmap;
   cudaError_t err = uses_tma(NV4) ? encode_row_tmap(a.X, a.n, a.d, &tmap) : zero_tmap(&tmap);
   if (err != cudaSuccess) return err;
-  int dev = 0, sms = 0, per_sm = 0;
-  cudaGetDevice(&dev);
-  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   err = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kSearchWarps * 32, smem);
   if (err != cudaSuccess) return err;
   int64_t blocks = (a.nq + kSearchWarps - 1) / kSearchWarps;
@@ -106,13 +148,83 @@ static cudaError_t launch_t(const SearchLaunch& a, cudaStream_t s) {
   if (err != cudaSuccess) return err;
   kern<<<dim3(unsigned(blocks)), kSearchWarps * 32, smem, s>>>(
       g, a.Q, a.nq, a.k, a.l, a.e, a.entry, a.out_ids, a.out_dists, a.stats, a.ticket, a.entries,
-      tmap);
+      wrows, tmap);
+  count_launch();
+  return cudaGetLastError();
+}
+
+// Wide rows (d > 256): a warp group per query (search_group.cuh).  The rows per
+// TMA round R are picked as for the one-warp form (largest R <= 8 that holds the
+// batch in one wave).  GANNS_WIDE_GROUP=0 selects the one-warp form (A/B knob).
+static bool wide_group_enabled() {
+  static const bool on = [] {
+    const char* e = std::getenv("GANNS_WIDE_GROUP");
+    return !(e && e[0] == '0');
+  }();
+  return on;
+}
+
+template <int CG, int TPL, bool L2>
+static cudaError_t launch_group_t(const SearchLaunch& a, cudaStream_t s) {
+  auto kern = search_group_kernel<CG, TPL, L2>;
+  static bool attr_done = false;
+  if (!attr_done) {
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         227 * 1024);
+    if (e == cudaSuccess)
+      e = cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+    if (e != cudaSuccess) return e;
+    attr_done = true;
+  }
+  int dev = 0, sms = 0, per_sm = 0;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  const int d4 = a.d / 4;
+  auto smem_for = [&](int r) {
+    return warp_smem_bytes(a.l, TPL, 8, d4, 1, r) + group_area_bytes();
+  };
+  static const int forced = [] {
+    const char* e = std::getenv("GANNS_WIDE_ROWS");
+    return e ? std::atoi(e) : 0;
+  }();
+  int wrows = kWideStageRows;
+  if (forced >= 1 && forced <= kWideStageRows) {
+    wrows = forced;
+  } else {
+    for (int r = kWideStageRows; r >= 4; --r) {
+      if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kGroupWarps * 32,
+                                                        smem_for(r)) != cudaSuccess)
+        break;
+      if (int64_t(per_sm) * sms >= a.nq) {
+        wrows = r;
+        break;
+      }
+    }
+  }
+  const size_t smem = smem_for(wrows);
+  if (smem > 227 * 1024) return cudaErrorInvalidValue;
+  GraphView g{a.nbr, a.X, nullptr, a.n, a.d_max, d4, a.metric};
+  cudaError_t err = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kGroupWarps * 32, smem);
+  if (err != cudaSuccess) return err;
+  int64_t blocks = a.nq;
+  const int64_t resident = int64_t(sms) * (per_sm > 0 ? per_sm : 1);
+  if (blocks > resident) blocks = resident;
+  err = cudaMemsetAsync(a.ticket, 0, sizeof(int32_t), s);
+  if (err != cudaSuccess) return err;
+  kern<<<dim3(unsigned(blocks)), kGroupWarps * 32, smem, s>>>(
+      g, a.Q, a.nq, a.k, a.l, a.e, a.entry, a.out_ids, a.out_dists, a.stats, a.ticket, a.entries,
+      wrows);
   count_launch();
   return cudaGetLastError();
 }
 
 template <int NV4, int TPL>
 static cudaError_t launch_m(const SearchLaunch& a, cudaStream_t s) {
+#if GANNS_NV4 >= 4
+  if (wide_group_enabled())
+    return a.metric == 0 ? launch_group_t<NV4 / 4, TPL, true>(a, s)
+                         : launch_group_t<NV4 / 4, TPL, false>(a, s);
+#endif
 #ifdef GANNS_DEV_ONE
   return launch_t<NV4, TPL, true>(a, s);
 #endif

@@ -199,3 +199,45 @@ def test_offset_ids():
     t = cu(a)
     g.offset_ids(t, 1000)
     assert t.cpu().numpy().tolist() == [1000, 1005, -1, 1007]
+
+
+# ------------------------------------- wide form (d > 256): rows per TMA round
+_WIDE_CHILD = r"""
+import sys, numpy as np, torch
+sys.path.insert(0, {root!r})
+import oracle, ganns_synth as syn, paper_conf_icde_yuwzqzl22_b200 as g
+cases = [(960, 32, "l2", 300), (384, 48, "ip", 300), (512, 100, "l2", 300), (960, 32, "l2", 3000)]
+for d, d_max, metric, nq in cases:
+    X = syn.random_int_points(2000, d, 0, 15, d + d_max)
+    Q = syn.random_int_points(nq, d, 0, 15, 7 * d)
+    nbr = syn.random_graph(2000, d_max, seed=d_max + d, min_degree=d_max // 2)
+    nbr[5:2000:3] = -1          # empty rows: explorations with no neighbour
+    graph = g.from_adjacency(nbr, d, metric)
+    for l in (16, 64):
+        ids, dists, st = g.search(graph, torch.from_numpy(X).cuda(), torch.from_numpy(Q).cuda(),
+                                  10, l, stats=True)
+        oi, od, os_ = oracle.search(nbr, X, Q, 10, l, metric=metric, threads=8, stats=True)
+        assert (ids.cpu().numpy() == oi).all(), (d, d_max, l)
+        assert (dists.cpu().numpy() == od).all(), (d, d_max, l)
+        assert (st.cpu().numpy()[:, :2] == os_[:, :2]).all(), (d, d_max, l)
+print("ok")
+"""
+
+
+@pytest.mark.parametrize("group", ["1", "0"])
+@pytest.mark.parametrize("rows", [1, 3, 5, 7, 8])
+def test_search_parity_wide_rows_per_round(group, rows):
+    """Wide rows (d > 256) run on a warp group per query (GANNS_WIDE_GROUP=1, the
+    default) or one warp (=0), staging R rows per TMA round (the launcher lowers R
+    so a small batch fits one wave).  Every form and R in 1..8 must give the
+    oracle's results bit for bit, including explorations of empty rows and
+    several queries per persistent CTA.  Knobs are read once, so each
+    combination runs in a child process."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, GANNS_WIDE_ROWS=str(rows), GANNS_WIDE_GROUP=group)
+    r = subprocess.run([sys.executable, "-c", _WIDE_CHILD.format(root=root)], env=env,
+                       capture_output=True, text=True, timeout=900)
+    assert r.returncode == 0 and r.stdout.strip().endswith("ok"), r.stderr[-3000:]
