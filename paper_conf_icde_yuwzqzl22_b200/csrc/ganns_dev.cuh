@@ -127,11 +127,6 @@ struct GraphView {
   int d_max;
   int d4;               // d / 4
   int metric;           // 0 L2, 1 IP, 2 COSINE
-  // L2 residency hint (0 = none): vector rows of vertices < hot are fetched with
-  // an evict_last policy (the early-inserted hubs every search passes through),
-  // the others with evict_first when cold_first is set
-  int32_t hot = 0;
-  int32_t cold_first = 0;
 };
 
 // Per-search counters (kept in registers, identical to the oracle's stats[0,1,3]).
@@ -377,23 +372,7 @@ __device__ __forceinline__ float tma_dot(const GraphView& g, const float4 (&qv)[
       __syncwarp();
       char* dst = reinterpret_cast<char*>(ws.stage) + size_t(my_slot) * rowbytes;
       if (issuer) {
-        if (g4 && g.hot > 0) {
-          // absent rows carry 0x7fffffff: never hot
-          const bool hot4 = uo < g.hot || u1 < g.hot || u2 < g.hot || u3 < g.hot;
-          uint64_t pol;
-          if (hot4)
-            asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
-          else if (g.cold_first)
-            asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
-          else
-            asm("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(pol));
-          asm volatile(
-              "cp.async.bulk.tensor.2d.shared::cta.global.tile::gather4.mbarrier::complete_tx::bytes"
-              ".L2::cache_hint [%0], [%1, {%2, %3, %4, %5, %6}], [%7], %8;" ::"r"(smem_u32(dst)),
-              "l"(g.tmap), "r"(0), "r"(uo), "r"(u1), "r"(u2), "r"(u3), "r"(smem_u32(ws.mbar)),
-              "l"(pol)
-              : "memory");
-        } else if (g4)
+        if (g4)
           asm volatile(
               "cp.async.bulk.tensor.2d.shared::cta.global.tile::gather4.mbarrier::complete_tx::bytes"
               " [%0], [%1, {%2, %3, %4, %5, %6}], [%7];" ::"r"(smem_u32(dst)),

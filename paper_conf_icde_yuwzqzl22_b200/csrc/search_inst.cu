@@ -123,19 +123,6 @@ static cudaError_t launch_t(const SearchLaunch& a, cudaStream_t s) {
     smem += size_t(pad);
   }
   GraphView g{a.nbr, a.X, nullptr, a.n, a.d_max, a.d / 4, a.metric};
-  {
-    // developer knobs (L2 residency experiments): GANNS_L2_HOT_ROWS, GANNS_L2_COLD_FIRST
-    static const int hot = [] {
-      const char* e = std::getenv("GANNS_L2_HOT_ROWS");
-      return e ? std::atoi(e) : 0;
-    }();
-    static const int cold_first = [] {
-      const char* e = std::getenv("GANNS_L2_COLD_FIRST");
-      return e ? std::atoi(e) : 0;
-    }();
-    g.hot = hot;
-    g.cold_first = cold_first;
-  }
   CUtensorMap tmap;
   cudaError_t err = uses_tma(NV4) ? encode_row_tmap(a.X, a.n, a.d, &tmap) : zero_tmap(&tmap);
   if (err != cudaSuccess) return err;
