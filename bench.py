@@ -77,29 +77,39 @@ class ClockSampler:
         self.stop = threading.Event()
         self.max_mhz = None
 
-    def _run(self):
+    def sample_now(self):
+        """One sample from the calling thread (bench loops call it between timed
+        steps, so a short timed region still has samples)."""
+        if getattr(self, "h", None) is None:
+            return
         import pynvml as nv
-        h = nv.nvmlDeviceGetHandleByIndex(self.index)
-        self.max_mhz = float(nv.nvmlDeviceGetMaxClockInfo(h, nv.NVML_CLOCK_SM))
+        try:
+            sm = float(nv.nvmlDeviceGetClockInfo(self.h, nv.NVML_CLOCK_SM))
+            rs = int(nv.nvmlDeviceGetCurrentClocksEventReasons(self.h))
+        except Exception:
+            return
+        self.samples.append((sm, rs))
+
+    def _run(self):
         while not self.stop.is_set():
-            try:
-                sm = float(nv.nvmlDeviceGetClockInfo(h, nv.NVML_CLOCK_SM))
-                rs = int(nv.nvmlDeviceGetCurrentClocksEventReasons(h))
-            except Exception:
+            n = len(self.samples)
+            self.sample_now()
+            if len(self.samples) == n:
                 break
-            self.samples.append((sm, rs))
             time.sleep(0.002)
 
     def __enter__(self):
+        self.h, self.t = None, None
         try:
             import pynvml as nv
             nv.nvmlInit()
             vis = os.environ.get("CUDA_VISIBLE_DEVICES")
             if vis:
                 self.index = int(vis.split(",")[self.index])
+            self.h = nv.nvmlDeviceGetHandleByIndex(self.index)
+            self.max_mhz = float(nv.nvmlDeviceGetMaxClockInfo(self.h, nv.NVML_CLOCK_SM))
             self.t = threading.Thread(target=self._run, daemon=True)
             self.t.start()
-            time.sleep(0.01)
         except Exception:
             self.t = None
         return self
@@ -331,6 +341,7 @@ def run_ours(args):
             e0.record(stream)
             index.search(Qd, k, l_star, e=e_star, out=out)
             e1.record(stream)
+            clk.sample_now()   # the step is running on the device
             e1.synchronize()
             times.append(e0.elapsed_time(e1))
     torch.cuda.synchronize()
@@ -528,6 +539,7 @@ def run_sharded(args):
             e0.record()
             ids, _ = step(l_star, l_star, ev=sev)
             e1.record()
+            clk.sample_now()
             e1.synchronize()
             times.append(e0.elapsed_time(e1) / 1e3)
     launches = g.kernel_launches() - launches0

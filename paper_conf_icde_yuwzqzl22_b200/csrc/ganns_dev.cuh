@@ -181,6 +181,12 @@ struct WarpSmem {
   int* pool_owner;          // -1 = free
   uint32_t* pool_phase;     // parity of each buffer's next phase
   int held;                 // buffer held by this warp, -1 = none
+  // stage pairing (search kernel, 2 warps per CTA, 2-round form): the CTA's two
+  // stages are contiguous at pair_stage; once the sibling warp has left (*pair_flag
+  // != 0) this warp switches to 1 round of 32 rows over both stages -- one memory
+  // round trip per exploration for the last queries of a batch
+  float4* pair_stage;
+  volatile int* pair_flag;
 };
 // Per-CTA layout of the pooled search kernel: [pool stages][per-warp N/T/bitmap][pool meta]
 __host__ __device__ constexpr size_t pooled_warp_bytes(int l, int tpl) {
@@ -204,6 +210,8 @@ __device__ __forceinline__ WarpSmem carve_warp_smem(uint8_t* base, int l, int tp
   w.phase = 0;
   w.pool = 0;
   w.held = -1;
+  w.pair_stage = nullptr;
+  w.pair_flag = nullptr;
   return w;
 }
 // pooled layout: warp w of `warps`; lane 0 of warp 0 initialises the pool
@@ -228,6 +236,8 @@ __device__ __forceinline__ WarpSmem carve_pooled_smem(uint8_t* cta, int w, int w
   s.stage = nullptr;
   s.phase = 0;
   s.held = -1;
+  s.pair_stage = nullptr;
+  s.pair_flag = nullptr;
   return s;
 }
 // acquire a free pool buffer (lane 0 spins on the owner words), make it current
@@ -546,6 +556,15 @@ struct WarpDist {
   }
   __device__ __forceinline__ float operator()(const GraphView& g, int32_t u_mine, int lane,
                                               WarpSmem& ws) {
+    if constexpr (uses_tma(NV4))
+      if (ws.pair_flag != nullptr && ws.rounds == 2) {
+        int f = 0;
+        if (lane == 0) f = atomicAdd(const_cast<int*>(ws.pair_flag), 0);   // atomic: orders the handover
+        if (__shfl_sync(kFull, f, 0) != 0) {
+          ws.rounds = 1;
+          ws.stage = ws.pair_stage;
+        }
+      }
     return group_distances<NV4, L2>(g, qv, u_mine, cbase, qinv, lane, ws);
   }
 };

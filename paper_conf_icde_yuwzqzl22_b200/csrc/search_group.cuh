@@ -14,8 +14,8 @@
 //     CTA's stage, and every warp of the group reduces its own slice of the
 //     columns (warp w owns float4 columns w*32 + lane + 32*G*f) for every staged
 //     row; per-warp row partials meet in shared memory and the leader adds them.
-// Commands pass through shared memory behind named barriers (bar.sync 1: a
-// command is published; bar.sync 2: a round's partials are written and the stage
+// Commands pass through shared memory behind named barriers (barrier 1: a
+// command is published; barrier 2: a round's partials are written and the stage
 // may be refilled).  Results are those of the one-warp search: the same N after
 // every iteration (distances are exact on integer-grid inputs whatever the
 // summation order, R-C18; cosine to rounding).
@@ -48,8 +48,12 @@ __device__ __forceinline__ GroupShared carve_group(uint8_t* p) {
   s.sQ = reinterpret_cast<int64_t*>(s.sCmd + 8);
   return s;
 }
+// Non-.aligned form: the leader and the helpers reach a barrier through different
+// barrier instructions (bar.sync is barrier.sync.aligned, which requires the same
+// instruction in every thread).
 __device__ __forceinline__ void group_bar(int id) {
-  asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(kGroupWarps * 32) : "memory");
+  __syncwarp();
+  asm volatile("barrier.sync %0, %1;" ::"r"(id), "r"(kGroupWarps * 32) : "memory");
 }
 
 // Query slice of warp w: float4 columns w*32 + lane + 32*G*f, f < CG.

@@ -13,6 +13,14 @@
 
 namespace ganns {
 
+#ifndef GANNS_PAIR_STAGES
+#define GANNS_PAIR_STAGES 1
+#endif
+// 2 warps per CTA, 2-round form: a warp whose sibling has left takes over both
+// stages (1 round per exploration) -- shortens the drain of a batch
+constexpr bool kPairStages = GANNS_PAIR_STAGES != 0 && GANNS_SEARCH_WARPS == 2 &&
+                             GANNS_SEARCH_ROUNDS == 2 && GANNS_SEARCH_POOL == 0;
+
 // Persistent: every warp pulls queries from a per-launch ticket counter until
 // the batch is exhausted, so the last wave is balanced at query granularity.
 template <int NV4, int TPL, bool L2>
@@ -35,6 +43,18 @@ search_kernel(GraphView g, const float* __restrict__ Q, int64_t nq, int k, int l
       ws.pool_phase[lane] = 0;
     }
     __syncthreads();
+  } else if (kPairStages && uses_tma(NV4)) {
+    // [stage 0][stage 1][warp 0: N/T/mbar/bitmap][warp 1: ...][flag]
+    const size_t sb = stage_bytes(NV4, g.d4, kSearchStageRounds);
+    const size_t rb = warp_smem_bytes(l, TPL, NV4, g.d4, kSearchStageRounds) - sb;
+    uint8_t* mine = smem + 2 * sb + size_t(w) * rb - sb;   // carve puts N right after the stage
+    ws = carve_warp_smem(mine, l, TPL, NV4, g.d4, kSearchStageRounds);
+    ws.stage = reinterpret_cast<float4*>(smem + size_t(w) * sb);
+    ws.pair_stage = reinterpret_cast<float4*>(smem);
+    ws.pair_flag = reinterpret_cast<volatile int*>(smem + 2 * sb + 2 * rb);
+    if (threadIdx.x == 0) *ws.pair_flag = 0;
+    if (lane == 0) mbar_init(ws.mbar, 1);
+    __syncthreads();
   } else {
     ws = carve_warp_smem(
         smem + size_t(w) * warp_smem_bytes(l, TPL, NV4, g.d4, kSearchStageRounds, wrows), l, TPL,
@@ -47,7 +67,11 @@ search_kernel(GraphView g, const float* __restrict__ Q, int64_t nq, int k, int l
   int32_t qt = 0;
   if (lane == 0) qt = atomicAdd(ticket, 1);
   const int64_t q = __shfl_sync(kFull, qt, 0);
-  if (q >= nq) break;
+  if (q >= nq) {
+    // this warp's stage is idle from now on: the sibling may take it over
+    if (ws.pair_flag != nullptr && lane == 0) atomicExch(const_cast<int*>(ws.pair_flag), 1);
+    break;
+  }
   SearchStats st;
   const int32_t ent = entries != nullptr ? entries[q] : entry;   // HNSW: per-query entry
   const int cnt = warp_search<NV4, TPL, L2, false>(g, Q + size_t(q) * (g.d4 * 4), ent, l, e,
@@ -112,7 +136,8 @@ static cudaError_t launch_t(const SearchLaunch& a, cudaStream_t s) {
                     ? pooled_cta_bytes(a.l, TPL, NV4, a.d / 4, kSearchStageRounds, kSearchWarps,
                                        kSearchPool)
                     : size_t(kSearchWarps) *
-                          warp_smem_bytes(a.l, TPL, NV4, a.d / 4, kSearchStageRounds, wrows);
+                          warp_smem_bytes(a.l, TPL, NV4, a.d / 4, kSearchStageRounds, wrows) +
+                          (kPairStages && uses_tma(NV4) ? 16 : 0);
   if (smem > 227 * 1024) return cudaErrorInvalidValue;
   {
     // developer knob (occupancy experiments): extra shared memory per CTA
