@@ -157,11 +157,26 @@ __host__ __device__ constexpr size_t stage_bytes(int nv4, int d4, int rounds,
                                                  int wrows = kWideStageRows) {
   return uses_tma(nv4) ? size_t(32 / rounds) * d4 * 16 : size_t(wrows) * d4 * 16;
 }
+// T (the surviving visiting entries, written and read only by the merge) lives
+// in the stage: the stage is idle from the end of an exploration's distance math
+// to the next exploration's first TMA round (whose issue is preceded by a
+// proxy fence).  The stage region is therefore at least T's size.
+__host__ __device__ constexpr size_t t_bytes(int tpl) { return size_t(tpl) * 32 * 8; }
+__host__ __device__ constexpr size_t stage_region_bytes(int nv4, int d4, int rounds, int tpl,
+                                                        int wrows = kWideStageRows) {
+  return stage_bytes(nv4, d4, rounds, wrows) > t_bytes(tpl) ? stage_bytes(nv4, d4, rounds, wrows)
+                                                           : t_bytes(tpl);
+}
+// the rest of a warp's area: N (lpad32(l) keys), the mbarrier (16 B), the merge
+// bitmap (lpad32(l) bits, 16-B rounded); a multiple of 16 B
+__host__ __device__ constexpr size_t warp_tail_bytes(int l) {
+  return size_t(lpad32(l)) * 8 + 16 + ((size_t(lpad32(l) / 32) * 4 + 15) & ~size_t(15));
+}
 __host__ __device__ constexpr size_t warp_smem_bytes(int l, int tpl, int nv4, int d4, int rounds,
                                                      int wrows = kWideStageRows) {
   // rounded to 128 B: the stage (first) must be 128-B aligned for tensor TMA
-  return (stage_bytes(nv4, d4, rounds, wrows) + size_t(lpad32(l)) * 8 + size_t(tpl) * 32 * 8 + 16 +
-          128 + 127) & ~size_t(127);
+  return (stage_region_bytes(nv4, d4, rounds, tpl, wrows) + warp_tail_bytes(l) + 127) &
+         ~size_t(127);
 }
 struct WarpSmem {
   float4* stage;
@@ -197,16 +212,20 @@ __host__ __device__ constexpr size_t pooled_cta_bytes(int l, int tpl, int nv4, i
   return size_t(pool) * stage_bytes(nv4, d4, rounds) + size_t(warps) * pooled_warp_bytes(l, tpl) +
          size_t(pool) * 16;
 }
+// N, mbarrier and bitmap of a warp at `tail` (16-B aligned, warp_tail_bytes(l))
+__device__ __forceinline__ void carve_warp_tail(WarpSmem& w, uint8_t* tail, int l) {
+  w.sN = reinterpret_cast<uint64_t*>(tail);
+  w.mbar = w.sN + lpad32(l);
+  w.sBM = reinterpret_cast<uint32_t*>(w.mbar + 2);
+}
 __device__ __forceinline__ WarpSmem carve_warp_smem(uint8_t* base, int l, int tpl, int nv4, int d4,
                                                    int rounds, int wrows = kWideStageRows) {
   WarpSmem w;
   w.rounds = rounds;
   w.wrows = wrows;
   w.stage = reinterpret_cast<float4*>(base);
-  w.sN = reinterpret_cast<uint64_t*>(base + stage_bytes(nv4, d4, rounds, wrows));
-  w.sT = w.sN + lpad32(l);
-  w.mbar = w.sT + tpl * 32;
-  w.sBM = reinterpret_cast<uint32_t*>(w.mbar + 2);
+  w.sT = reinterpret_cast<uint64_t*>(base);   // shares the stage (see t_bytes)
+  carve_warp_tail(w, base + stage_region_bytes(nv4, d4, rounds, tpl, wrows), l);
   w.phase = 0;
   w.pool = 0;
   w.held = -1;
@@ -651,6 +670,7 @@ __device__ int warp_search_with(const GraphView& g, DIST& dist, int32_t entry, i
       key[t] = u[t] >= 0 ? mkkey(dd, u[t]) : kKeyInf;
       st.comps += __popc(__ballot_sync(kFull, u[t] >= 0));
     }
+    __syncwarp();   // every lane's stage reads precede the merge's writes of T (it shares the stage)
     // (4) lazy check (R-C1): drop entries already in N; entries that
     // cannot enter N (>= its l-th key while N is full) are dropped as well.
     const uint64_t worst = cnt == l ? unflag(sN[l - 1]) : kKeyInf;

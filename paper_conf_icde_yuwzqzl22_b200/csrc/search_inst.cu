@@ -44,12 +44,12 @@ search_kernel(GraphView g, const float* __restrict__ Q, int64_t nq, int k, int l
     }
     __syncthreads();
   } else if (kPairStages && uses_tma(NV4)) {
-    // [stage 0][stage 1][warp 0: N/T/mbar/bitmap][warp 1: ...][flag]
-    const size_t sb = stage_bytes(NV4, g.d4, kSearchStageRounds);
-    const size_t rb = warp_smem_bytes(l, TPL, NV4, g.d4, kSearchStageRounds) - sb;
-    uint8_t* mine = smem + 2 * sb + size_t(w) * rb - sb;   // carve puts N right after the stage
-    ws = carve_warp_smem(mine, l, TPL, NV4, g.d4, kSearchStageRounds);
-    ws.stage = reinterpret_cast<float4*>(smem + size_t(w) * sb);
+    // [stage 0][stage 1][warp 0: N/mbar/bitmap][warp 1: ...][flag]; each stage
+    // region also holds its warp's T (ganns_dev.cuh: t_bytes)
+    const size_t sb = stage_region_bytes(NV4, g.d4, kSearchStageRounds, TPL);
+    const size_t rb = warp_tail_bytes(l);
+    ws = carve_warp_smem(smem + size_t(w) * sb, l, TPL, NV4, g.d4, kSearchStageRounds);
+    carve_warp_tail(ws, smem + 2 * sb + size_t(w) * rb, l);
     ws.pair_stage = reinterpret_cast<float4*>(smem);
     ws.pair_flag = reinterpret_cast<volatile int*>(smem + 2 * sb + 2 * rb);
     if (threadIdx.x == 0) *ws.pair_flag = 0;
@@ -135,9 +135,11 @@ static cudaError_t launch_t(const SearchLaunch& a, cudaStream_t s) {
   size_t smem = kSearchPool > 0
                     ? pooled_cta_bytes(a.l, TPL, NV4, a.d / 4, kSearchStageRounds, kSearchWarps,
                                        kSearchPool)
+                : kPairStages && uses_tma(NV4)
+                    ? 2 * (stage_region_bytes(NV4, a.d / 4, kSearchStageRounds, TPL) +
+                           warp_tail_bytes(a.l)) + 16
                     : size_t(kSearchWarps) *
-                          warp_smem_bytes(a.l, TPL, NV4, a.d / 4, kSearchStageRounds, wrows) +
-                          (kPairStages && uses_tma(NV4) ? 16 : 0);
+                          warp_smem_bytes(a.l, TPL, NV4, a.d / 4, kSearchStageRounds, wrows);
   if (smem > 227 * 1024) return cudaErrorInvalidValue;
   {
     // developer knob (occupancy experiments): extra shared memory per CTA

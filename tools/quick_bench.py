@@ -18,6 +18,8 @@ ap.add_argument("--l-build", type=int, default=0)
 ap.add_argument("--group", type=int, default=0)
 ap.add_argument("--reps", type=int, default=5)
 ap.add_argument("--nq-mult", default="1", help="comma list: time batches of m x nq queries")
+ap.add_argument("--orders", default="", help="comma list of pivot counts P: also time the batch "
+                "reordered by each query's nearest of P evenly spaced points (locality experiment)")
 a = ap.parse_args()
 cfg = syn.CONFIGS[a.config]
 X = torch.from_numpy(syn.points(cfg)).cuda()
@@ -58,6 +60,21 @@ for l in [int(x) for x in a.ls.split(",")]:
             tm.append(e0.elapsed_time(e1) / 1e3)
         tmm = sorted(tm)[len(tm) // 2]
         print(json.dumps({"l": l, "nq": len(Qm), "ms": round(tmm * 1e3, 3), "qps": round(len(Qm) / tmm)}))
+    for P in [int(x) for x in a.orders.split(",") if x]:
+        piv = X[:: max(1, len(X) // P)][:P]
+        lab = torch.cdist(Q, piv).argmin(1)
+        Qo = Q[torch.argsort(lab, stable=True)].contiguous()
+        to = []
+        for _ in range(a.reps):
+            flush.zero_()
+            e0, e1 = torch.cuda.Event(True), torch.cuda.Event(True)
+            e0.record()
+            g.search(graph, X, Qo, cfg.k, l)
+            e1.record()
+            e1.synchronize()
+            to.append(e0.elapsed_time(e1) / 1e3)
+        tom = sorted(to)[len(to) // 2]
+        print(json.dumps({"l": l, "order_pivots": P, "ms": round(tom * 1e3, 3), "qps": round(len(Q) / tom)}))
     print(json.dumps({"l": l, "recall": round(recall_at(ids, gt), 4), "ms": round(t * 1e3, 3),
                       "qps": round(len(Q) / t), "alg_GBps": round(byts / t / 1e9, 1),
                       "iters": round(float(st[:, 0].float().mean()), 1),
