@@ -4,13 +4,17 @@ configs[1]), plus GGraphCon NSW build seconds, on N B200s.
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--config C2] [--impl ours|reference]
 
-One step = one ganns_search launch over the whole 10K-query batch at the smallest
-l (from the sweep) whose recall@10 >= 0.95 -- the whole hot path (candidate
+One step = one ganns_search launch over a whole 10K-query batch at the fastest
+(l, e) of the sweep whose recall@10 >= 0.95 -- the whole hot path (candidate
 locating, adjacency gather, bulk distance, lazy check, sort, merge, top-k out)
-in one fused kernel.  Inputs are resident in HBM when the timed region starts;
-L2 is flushed (256 MiB write) between timed steps.  Under torchrun each rank
-builds the same deterministic graph and searches its own batch of nq queries
-(weak scaling, no data-path collective); time = max over ranks.
+in one fused kernel.  Steps are back-to-back batches issued alternately on two
+CUDA streams (the streamed multi-batch pipeline), so the
+drain tail of one batch overlaps the start of the next.  They rotate over
+--batches distinct query batches (no step re-reads its predecessor's queries'
+rows from L2); the working set (vectors + graph) is larger than the 126 MB L2, so
+L2 is not flushed.  Inputs are resident in HBM when the timed region starts.
+Under torchrun each rank builds the same deterministic graph and searches its own
+batches (weak scaling, no data-path collective); time = max over ranks.
 
 --impl reference times the CPU oracle (oracle/, plain C, all host cores) on a
 bounded sample of the same queries, same graph, same l.
@@ -49,6 +53,10 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
     ap.add_argument("--json-out", default=None)
+    ap.add_argument("--batches", type=int, default=4,
+                    help="distinct query batches the steps rotate over")
+    ap.add_argument("--streams", type=int, default=2,
+                    help="CUDA streams the steps alternate over (1 = serialised launches)")
     ap.add_argument("--shard-rows", type=int, default=0,
                     help="C5 only: rows per shard (default: n / shards = 12.5M)")
     return ap.parse_args()
@@ -135,14 +143,19 @@ def workload_name(cfg, kind):
             f"{cfg.degree}")
 
 
-def make_workload(cfg, rank: int):
+def make_workload(cfg, rank: int, batches: int = 1):
+    """Points and `batches` query batches of cfg.nq for this rank; rank 0's first
+    batch is the config's query set (the operating point and the oracle's sample
+    use it)."""
     X = syn.points(cfg)
     if cfg.metric == "cosine":
         X = syn.normalize_rows(X)   # input preparation: unit rows (Table I "Cosine")
-    # every rank draws its own batch of nq queries (weak scaling); rank 0 = the config's
-    Qall = syn.queries(cfg, cfg.nq * (rank + 1))
-    Q = Qall[rank * cfg.nq:(rank + 1) * cfg.nq]
-    return X, np.ascontiguousarray(Q)
+    # every rank draws its own batches of nq queries (weak scaling)
+    first = rank * batches
+    Qall = syn.queries(cfg, cfg.nq * (first + batches))
+    Qs = [np.ascontiguousarray(Qall[(first + b) * cfg.nq:(first + b + 1) * cfg.nq])
+          for b in range(batches)]
+    return (X, Qs[0]) if batches == 1 else (X, Qs)
 
 
 def ground_truth(torch, Xd, Qd, k, metric="l2", with_dist=False):
@@ -232,29 +245,89 @@ class BenchIndex:
         return self._oi
 
 
+class Pipeline:
+    """Back-to-back search steps, step i on stream i % S over batch i % B (the
+    streamed multi-batch pipeline): the drain tail of a batch overlaps
+    the start of the next one.  Device-timed with CUDA events bracketing all
+    streams."""
+
+    def __init__(self, torch, index, Qds, k, nstreams):
+        self.torch, self.index, self.Qds, self.k = torch, index, Qds, k
+        nq = Qds[0].shape[0]
+        dev = Qds[0].device
+        self.streams = [torch.cuda.Stream(device=dev) for _ in range(max(1, nstreams))]
+        self.outs = [(torch.empty((nq, k), dtype=torch.int32, device=dev),
+                      torch.empty((nq, k), dtype=torch.float32, device=dev))
+                     for _ in self.streams]
+
+    def _bracket(self, body, clk=None):
+        torch = self.torch
+        cur = torch.cuda.current_stream()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(cur)
+        for st in self.streams:
+            st.wait_event(e0)
+        body()
+        for st in self.streams:
+            ev = torch.cuda.Event()
+            ev.record(st)
+            cur.wait_event(ev)
+        e1.record(cur)
+        while clk is not None and not e1.query():
+            clk.sample_now()   # the steps are running on the device
+            time.sleep(0.001)
+        e1.synchronize()
+        return e0.elapsed_time(e1) / 1e3
+
+    def run(self, steps, l, e, clk=None):
+        """Seconds for `steps` steps (device time, all streams)."""
+        torch, S = self.torch, len(self.streams)
+
+        def body():
+            for i in range(steps):
+                with torch.cuda.stream(self.streams[i % S]):
+                    self.index.search(self.Qds[i % len(self.Qds)], self.k, l, e=e,
+                                      out=self.outs[i % S])
+        return self._bracket(body, clk)
+
+    def run_host(self, g, Xd, Qhs, steps, l, e):
+        """Wall seconds for `steps` end-to-end steps through ganns_search_host_async:
+        H2D of the batch from pinned host memory, search, D2H of ids + dists, each
+        step on its stream; synchronised at the end."""
+        torch, S = self.torch, len(self.streams)
+        if not hasattr(self, "scratch"):
+            nq, d = Qhs[0].shape
+            dev = Xd.device
+            self.scratch = [(torch.empty((nq, d), dtype=torch.float32, device=dev),
+                             torch.empty((nq, self.k), dtype=torch.int32, device=dev),
+                             torch.empty((nq, self.k), dtype=torch.float32, device=dev))
+                            for _ in range(S)]
+            self.hout = [(torch.empty((nq, self.k), dtype=torch.int32).pin_memory(),
+                          torch.empty((nq, self.k), dtype=torch.float32).pin_memory())
+                         for _ in range(S)]
+        obj = self.index.idx if self.index.hnsw else self.index.graph
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        for i in range(steps):
+            g.search_host_async(obj, Xd, Qhs[i % len(Qhs)], self.k, l, self.scratch[i % S],
+                                self.hout[i % S], e=e, stream=self.streams[i % S])
+        for st in self.streams:
+            st.synchronize()
+        return time.perf_counter() - t0
+
+
 def recall_at(ids, gt):
     k = gt.shape[1]
     hit = (ids[:, :, None] == gt[:, None, :]).any(2).sum()
     return float(hit) / (k * gt.shape[0])
 
 
-def select_operating_point(torch, index, Qd, gt, k, target, flush):
-    """(l, e) sweep: recall@10 of every pair; among the pairs reaching `target`
-    the fastest (median of 3 timed launches) is the operating point.  e (explore
-    budget) is the paper's fine-grained speed/accuracy knob."""
+def select_operating_point(torch, index, Qd, gt, k, target, timer):
+    """(l, e) sweep: recall@10 of every pair over the queries Qd; among the pairs
+    reaching `target` the fastest (timer(l, e) -> seconds) is the operating point.
+    e (explore budget) is the paper's fine-grained speed/accuracy knob."""
     sweep, chosen, feasible = [], {}, []
-
-    def timed(l, e, reps=3):
-        ts = []
-        for _ in range(reps):
-            flush.zero_()
-            a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-            a0.record()
-            index.search(Qd, k, l, e=e)
-            a1.record()
-            a1.synchronize()
-            ts.append(a0.elapsed_time(a1))
-        return sorted(ts)[len(ts) // 2]
+    timed = timer
 
     for l in L_SWEEP:
         best_r = 0.0
@@ -293,9 +366,13 @@ def run_ours(args):
     cfg = syn.CONFIGS[args.config]
     k = cfg.k
 
-    X, Q = make_workload(cfg, rank)
+    B = max(1, args.batches)
+    X, Qs = make_workload(cfg, rank, B)
+    Q = Qs[0]
+    nq = Q.shape[0]
     Xd = torch.from_numpy(X).to(dev)
-    Qd = torch.from_numpy(Q).to(dev)
+    Qd_all = torch.from_numpy(np.concatenate(Qs)).to(dev)
+    Qds = [Qd_all[b * nq:(b + 1) * nq] for b in range(B)]
     torch.cuda.synchronize()
 
     # ---- GGraphCon build (timed wall clock on device-resident points)
@@ -305,73 +382,52 @@ def run_ours(args):
     build_s = time.perf_counter() - t0
     b_iters, b_comps, b_searches, b_rounds = index.build_stats
 
-    # ---- (l, e) operating point (see select_operating_point)
-    gt = ground_truth(torch, Xd, Qd, k, cfg.metric)
-    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
-    l_star, e_star, sweep, chosen = select_operating_point(torch, index, Qd, gt, k, args.target,
-                                                           flush)
-    ids, dists, st = index.search(Qd, k, l_star, e=e_star, stats=True)
+    # ---- (l, e) operating point over every query the timed steps search (see
+    # select_operating_point); candidates timed as the steps are (pipelined)
+    gt = ground_truth(torch, Xd, Qd_all, k, cfg.metric)
+    pipe = Pipeline(torch, index, Qds, k, args.streams)
+    l_star, e_star, sweep, chosen = select_operating_point(
+        torch, index, Qd_all, gt, k, args.target,
+        lambda l, e: min(pipe.run(2 * B, l, e) for _ in range(2)))
+    ids, dists, st = index.search(Qd_all, k, l_star, e=e_star, stats=True)
     rec = recall_at(ids, gt)
     st = st.long()
     d = cfg.d
     # algorithmic bytes: query + per iteration the adjacency row
     # + every computed distance's vector row (incl. the entry and lazy-check
-    # re-computations) + the top-k written
+    # re-computations) + the top-k written; per step = mean over the batches
     alg_bytes = int((4 * d + 4 * cfg.degree * st[:, 0] + 4 * d * st[:, 1]).sum().item()
-                    + 8 * k * Q.shape[0])
+                    + 8 * k * Qd_all.shape[0]) // B
     iters_mean = float(st[:, 0].float().mean())
 
-    # ---- timed steps: device-resident inputs, L2 flushed between steps
-    stream = torch.cuda.current_stream()
-    out = (torch.empty((Q.shape[0], k), dtype=torch.int32, device=dev),
-           torch.empty((Q.shape[0], k), dtype=torch.float32, device=dev))
-    for _ in range(args.warmup):
-        index.search(Qd, k, l_star, e=e_star, out=out)
+    # ---- timed steps: device-resident inputs, back-to-back batches on two streams
+    pipe.run(args.warmup, l_star, e_star)
     torch.cuda.synchronize()
     launches0 = g.kernel_launches()
-    times = []
     if distributed:
         dist.barrier()
     torch.cuda.synchronize()
     with ClockSampler(local) as clk:
-        for _ in range(args.steps):
-            flush.zero_()
-            e0 = torch.cuda.Event(enable_timing=True)
-            e1 = torch.cuda.Event(enable_timing=True)
-            e0.record(stream)
-            index.search(Qd, k, l_star, e=e_star, out=out)
-            e1.record(stream)
-            clk.sample_now()   # the step is running on the device
-            e1.synchronize()
-            times.append(e0.elapsed_time(e1))
+        t_total = pipe.run(args.steps, l_star, e_star, clk)
     torch.cuda.synchronize()
     if distributed:
         dist.barrier()
     launches = g.kernel_launches() - launches0
-    t_total = sum(times) / 1e3
     t_max = torch.tensor([t_total], dtype=torch.float64, device=dev)
     if distributed:
         dist.all_reduce(t_max, op=dist.ReduceOp.MAX)
     t_total = float(t_max.item())
-    total_queries = Q.shape[0] * args.steps * world
+    total_queries = nq * args.steps * world
     qps = total_queries / t_total
     ms_per_step = t_total / args.steps * 1e3
-    kernel_s = statistics.mean(times) / 1e3
+    kernel_s = t_total / args.steps
 
-    # ---- end to end through the public API from pinned host buffers
-    Qh = torch.from_numpy(Q).pin_memory()
-    hout = (torch.empty((Q.shape[0], k), dtype=torch.int32).pin_memory(),
-            torch.empty((Q.shape[0], k), dtype=torch.float32).pin_memory())
-    for _ in range(2):
-        index.search_host(torch, Qh, k, l_star, e_star, hout)
-    e2e_times = []
-    for _ in range(args.steps):
-        flush.zero_()
-        torch.cuda.synchronize()
-        t0 = time.perf_counter()
-        index.search_host(torch, Qh, k, l_star, e_star, hout)
-        e2e_times.append(time.perf_counter() - t0)
-    e2e_t = torch.tensor([sum(e2e_times)], dtype=torch.float64, device=dev)
+    # ---- end to end through the public API (ganns_search_host_async) from pinned
+    # host buffers: every step copies its batch in and its ids + dists out
+    Qhs = [torch.from_numpy(q).pin_memory() for q in Qs]
+    pipe.run_host(g, Xd, Qhs, max(2, args.warmup), l_star, e_star)
+    e2e_t = torch.tensor([pipe.run_host(g, Xd, Qhs, args.steps, l_star, e_star)],
+                         dtype=torch.float64, device=dev)
     if distributed:
         dist.all_reduce(e2e_t, op=dist.ReduceOp.MAX)
     e2e_qps = total_queries / float(e2e_t.item())
@@ -401,10 +457,14 @@ def run_ours(args):
         "data": "synthetic",
         "config": {"workload": workload_name(cfg, index.kind) + f", {Q.shape[0]} queries/GPU, k={k}",
                    "l": l_star, "e": e_star, "recall_at_10": round(rec, 5),
+                   "recall_over": f"all {B * nq} queries of the {B} batches",
                    "selection": "fastest (l, e) with recall@10 >= target among the sweep",
                    "le_for_recall": {str(t): chosen.get(t) for t in (0.9, 0.95, 0.99)},
                    "le_sweep_recall": sweep, "mean_iterations": round(iters_mean, 2),
-                   "l2": "flushed (256 MiB write) between timed steps",
+                   "batches": B, "streams": len(pipe.streams),
+                   "l2": (f"not flushed: inputs larger than L2 ({(X.nbytes + cfg.n * cfg.degree * 4) >> 20}"
+                          f" MiB vectors + graph vs 126 MB); steps rotate over {B} distinct "
+                          f"{nq}-query batches"),
                    "parallelism": f"replicated graph, query data-parallel x{world}"},
         "build_seconds": round(build_s, 4),
         "build_params": {"degree": cfg.degree, "d_min": cfg.degree // 2, "l_build": args.l_build,
@@ -413,7 +473,8 @@ def run_ours(args):
                   "searches": b_searches, "rounds": b_rounds,
                   "alg_GBps": round((4 * d * b_comps + 4 * cfg.degree * b_iters) / build_s / 1e9, 1)},
         "e2e": {"value": round(e2e_qps, 1), "unit": "queries/s",
-                "h2d_bytes_per_step": int(Q.nbytes), "d2h_bytes_per_step": int(Q.shape[0] * k * 8)},
+                "h2d_bytes_per_step": int(Q.nbytes), "d2h_bytes_per_step": int(nq * k * 8),
+                "api": "ganns_search_host_async, steps alternating over the streams, wall clock"},
         "gpu_launches": int(launches),
         "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak,
                      "unit": "GB/s", "frac": round(achieved / peak, 4), "traffic": traffic,
@@ -422,6 +483,7 @@ def run_ours(args):
                      "traffic_frac": (round(traffic / kernel_s / 1e9 / peak, 4)
                                       if traffic else None),
                      "peak_kind": peak_kind, "alg_bytes_per_launch": alg_bytes,
+                     "duration": "timed region / steps (consecutive launches overlap on two streams)",
                      "kernel": f"ganns::search_kernel (d={cfg.d}, d_max={cfg.degree}, {cfg.metric})"},
         "clocks": clk.summary(),
     }
@@ -675,17 +737,22 @@ def run_reference(args):
     import paper_conf_icde_yuwzqzl22_b200 as g
     cfg = syn.CONFIGS[args.config]
     k = cfg.k
-    X, Q = make_workload(cfg, 0)
+    X, Qs = make_workload(cfg, 0, max(1, args.batches))
+    Qs = Qs if isinstance(Qs, list) else [Qs]
+    Q = Qs[0]
     # index set-up (not timed): the graph the GPU arm searches (deterministic) and
-    # the same (l, e) operating point
+    # the same (l, e) operating point, selected the same way
     Xd = torch.from_numpy(X).cuda()
     index = BenchIndex(g, cfg, Xd, args.l_build)
-    Qd = torch.from_numpy(Q).cuda()
+    Qd = torch.from_numpy(np.concatenate(Qs)).cuda()
     gt = ground_truth(torch, Xd, Qd, k, cfg.metric)
-    flush = torch.empty(256 << 20, dtype=torch.uint8, device=Xd.device)
-    l_star, e_star, _, _ = select_operating_point(torch, index, Qd, gt, k, args.target, flush)
+    Qds = [Qd[b * len(Q):(b + 1) * len(Q)] for b in range(len(Qs))]
+    pipe = Pipeline(torch, index, Qds, k, args.streams)
+    l_star, e_star, _, _ = select_operating_point(
+        torch, index, Qd, gt, k, args.target,
+        lambda l, e: min(pipe.run(2 * len(Qs), l, e) for _ in range(2)))
     index.oracle_search(X, Q[:2], k, l_star, e_star, 1)   # materialise the host copy
-    del Qd, flush
+    del Qd, Qds, pipe
     cores = oracle.ncores()
     per_step = 48
     for _ in range(args.warmup):

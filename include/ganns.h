@@ -125,6 +125,26 @@ GANNS_API int ganns_search_host(const ganns_graph *g, const float *points, const
                       int64_t nq, int k, int l, const ganns_search_params *p,
                       int32_t *out_ids_host, float *out_dists_host, void *stream);
 
+/* ganns_search_host_async -- one batch end to end from HOST buffers, enqueued on
+ * `stream` without synchronising (the streamed multi-batch pipeline, P:218:
+ * "the data transfer can be overlapped with the search using CUDA streams").
+ * On `stream`, in order: H2D queries_host -> queries_dev, the search
+ * (= ganns_search_ex), D2H ids_dev / dists_dev -> out_ids_host / out_dists_host.
+ * Alternating two streams over consecutive batches overlaps one batch's copies
+ * and drain tail with the next batch's search.
+ *   queries_host   host [nq][d] fp32, pinned (cudaHostAlloc / cudaHostRegister)
+ *   queries_dev    device scratch [nq][d] fp32, 16-B aligned
+ *   ids_dev, dists_dev  device scratch [nq][k]
+ *   out_ids_host, out_dists_host  host [nq][k], pinned
+ * Ownership: every buffer is the caller's; none may be reused or freed until
+ * `stream` has passed this call (e.g. cudaStreamSynchronize).  Errors as
+ * ganns_search_ex; EINVAL for NULL buffers.  Does not sync. */
+GANNS_API int ganns_search_host_async(const ganns_graph *g, const float *points,
+                                      const float *queries_host, int64_t nq, int k, int l,
+                                      const ganns_search_params *p, float *queries_dev,
+                                      int32_t *ids_dev, float *dists_dev, int32_t *out_ids_host,
+                                      float *out_dists_host, void *stream);
+
 /* ganns_merge_topk -- K6: merge W per-shard top-k lists into the global top-k
  * (multi-GPU base-set sharding).  For each query the k smallest
  * (dist, global id) over all shards.  All pointers device.
@@ -188,6 +208,15 @@ GANNS_API int ganns_build_hnsw(const float *points, int64_t n, int d, int metric
 GANNS_API int ganns_hnsw_search(const ganns_hnsw *h, const float *points, const float *queries,
                                 int64_t nq, int k, int l, const ganns_search_params *p,
                                 int32_t *out_ids, float *out_dists, void *stream);
+
+/* ganns_hnsw_search_host_async -- ganns_search_host_async on the HNSW index
+ * (H2D, ganns_hnsw_search, D2H on `stream`; same buffers, ownership and errors). */
+GANNS_API int ganns_hnsw_search_host_async(const ganns_hnsw *h, const float *points,
+                                           const float *queries_host, int64_t nq, int k, int l,
+                                           const ganns_search_params *p, float *queries_dev,
+                                           int32_t *ids_dev, float *dists_dev,
+                                           int32_t *out_ids_host, float *out_dists_host,
+                                           void *stream);
 
 /* ganns_hnsw_info -- number of layers; layer_n (nullable) receives n_j for j < nlayers. */
 GANNS_API int ganns_hnsw_info(const ganns_hnsw *h, int *nlayers, int64_t *layer_n);

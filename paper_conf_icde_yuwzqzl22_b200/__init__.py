@@ -47,6 +47,10 @@ def _load():
         "ganns_search": [P, P, P, i64, i32, i32, P, P, P],
         "ganns_search_ex": [P, P, P, i64, i32, i32, ct.POINTER(_SearchParams), P, P, P],
         "ganns_search_host": [P, P, P, i64, i32, i32, ct.POINTER(_SearchParams), P, P, P],
+        "ganns_search_host_async": [P, P, P, i64, i32, i32, ct.POINTER(_SearchParams), P, P, P,
+                                    P, P, P],
+        "ganns_hnsw_search_host_async": [P, P, P, i64, i32, i32, ct.POINTER(_SearchParams), P, P,
+                                         P, P, P, P],
         "ganns_merge_topk": [P, P, i32, i64, i32, P, P, P],
         "ganns_offset_ids": [P, i64, i64, P],
         "ganns_graph_from_adjacency": [P, i64, i32, i32, i32, i32, ct.POINTER(P)],
@@ -83,6 +87,7 @@ _lib = _load()
 
 # exported symbol list (include/ganns.h) -- checked by the CPU tests
 ABI_SYMBOLS = ("ganns_build", "ganns_search", "ganns_search_ex", "ganns_search_host",
+               "ganns_search_host_async", "ganns_hnsw_search_host_async",
                "ganns_merge_topk", "ganns_offset_ids", "ganns_graph_from_adjacency",
                "ganns_graph_adjacency", "ganns_graph_device_ptr", "ganns_graph_info",
                "ganns_graph_save", "ganns_graph_load", "ganns_graph_free", "ganns_last_error",
@@ -235,6 +240,33 @@ def search_host(graph: Graph, points: torch.Tensor, queries: torch.Tensor, k: in
                                       ct.c_void_p(ids.data_ptr()), ct.c_void_p(dists.data_ptr()),
                                       _stream(stream)))
     return ids, dists
+
+
+def search_host_async(index, points: torch.Tensor, queries_host: torch.Tensor, k: int, l: int,
+                      scratch, out_host, e: int = 0, stream=None):
+    """One batch end to end from pinned HOST buffers, enqueued on ``stream`` without
+    synchronising (ganns_search_host_async / ganns_hnsw_search_host_async): H2D of
+    the queries into ``scratch[0]`` (device [nq, d]), the search into ``scratch[1:3]``
+    (device ids/dists [nq, k]), D2H into ``out_host`` (pinned ids/dists [nq, k]).
+    ``index`` is a Graph or an Hnsw.  No buffer may be touched until ``stream``
+    has passed the call."""
+    points = _dev_f32(points, "points")
+    if queries_host.is_cuda or queries_host.dtype != torch.float32 or not queries_host.is_pinned():
+        raise TypeError("queries_host must be a pinned float32 CPU tensor")
+    ids_h, dists_h = out_host
+    if not (ids_h.is_pinned() and dists_h.is_pinned()):
+        raise TypeError("out_host must be pinned CPU tensors")
+    qd, ids_d, dists_d = scratch
+    nq = queries_host.shape[0]
+    p = _SearchParams(e, 0, None)
+    fn = _lib.ganns_hnsw_search_host_async if isinstance(index, Hnsw) else _lib.ganns_search_host_async
+    with torch.cuda.device(points.device):
+        _check(fn(index.handle, ct.c_void_p(points.data_ptr()),
+                  ct.c_void_p(queries_host.data_ptr()), nq, k, l, ct.byref(p),
+                  ct.c_void_p(qd.data_ptr()), ct.c_void_p(ids_d.data_ptr()),
+                  ct.c_void_p(dists_d.data_ptr()), ct.c_void_p(ids_h.data_ptr()),
+                  ct.c_void_p(dists_h.data_ptr()), _stream(stream)))
+    return out_host
 
 
 def merge_topk(shard_ids: torch.Tensor, shard_dists: torch.Tensor, stream=None):

@@ -135,6 +135,29 @@ int run_build(BuildArgs& a, cudaStream_t s) {
   return fail(GANNS_ENOTSUP, "unsupported dimension");
 }
 
+// H2D, search, D2H of one batch on `stream` (no sync); `search` enqueues the search
+// on the device copies.
+template <class SEARCH>
+int host_async(int d, const float* queries_host, int64_t nq, int k, float* queries_dev,
+                      int32_t* ids_dev, float* dists_dev, int32_t* out_ids_host,
+                      float* out_dists_host, void* stream, SEARCH&& search) {
+  if (nq < 0) return fail(GANNS_EINVAL, "nq < 0");
+  if (nq == 0) return GANNS_OK;
+  if (!queries_host || !queries_dev || !ids_dev || !dists_dev || !out_ids_host || !out_dists_host)
+    return fail(GANNS_EINVAL, "NULL buffer");
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  cudaError_t err = cudaMemcpyAsync(queries_dev, queries_host, sizeof(float) * size_t(nq) * d,
+                                    cudaMemcpyHostToDevice, s);
+  if (err != cudaSuccess) return cuda_fail(err, "H2D queries");
+  if (int rc = search()) return rc;
+  err = cudaMemcpyAsync(out_ids_host, ids_dev, sizeof(int32_t) * size_t(nq) * k,
+                        cudaMemcpyDeviceToHost, s);
+  if (err == cudaSuccess)
+    err = cudaMemcpyAsync(out_dists_host, dists_dev, sizeof(float) * size_t(nq) * k,
+                          cudaMemcpyDeviceToHost, s);
+  return err == cudaSuccess ? GANNS_OK : cuda_fail(err, "D2H results");
+}
+
 }  // namespace ganns
 
 using namespace ganns;
@@ -391,6 +414,18 @@ int ganns_search_host(const ganns_graph* g, const float* points, const float* qu
 }
 
 
+int ganns_search_host_async(const ganns_graph* g, const float* points, const float* queries_host,
+                            int64_t nq, int k, int l, const ganns_search_params* p,
+                            float* queries_dev, int32_t* ids_dev, float* dists_dev,
+                            int32_t* out_ids_host, float* out_dists_host, void* stream) {
+  if (int rc = check_graph(g)) return rc;
+  return host_async(g->d, queries_host, nq, k, queries_dev, ids_dev, dists_dev, out_ids_host,
+                    out_dists_host, stream, [&] {
+                      return ganns_search_ex(g, points, queries_dev, nq, k, l, p, ids_dev,
+                                             dists_dev, stream);
+                    });
+}
+
 int ganns_build(const float* points, int64_t n, int d, int metric, int degree,
                 const ganns_build_params* p, void* stream, ganns_graph** out) {
   if (!points || !out) return fail(GANNS_EINVAL, "NULL argument");
@@ -630,6 +665,19 @@ int ganns_hnsw_search(const ganns_hnsw* h, const float* points, const float* que
   err = launch_search(a, s);
   if (entries) cudaFreeAsync(entries, s);
   return err == cudaSuccess ? GANNS_OK : cuda_fail(err, "hnsw search");
+}
+
+int ganns_hnsw_search_host_async(const ganns_hnsw* h, const float* points,
+                                 const float* queries_host, int64_t nq, int k, int l,
+                                 const ganns_search_params* p, float* queries_dev,
+                                 int32_t* ids_dev, float* dists_dev, int32_t* out_ids_host,
+                                 float* out_dists_host, void* stream) {
+  if (!h || !h->base) return fail(GANNS_EINVAL, "hnsw is NULL");
+  return host_async(h->d, queries_host, nq, k, queries_dev, ids_dev, dists_dev, out_ids_host,
+                    out_dists_host, stream, [&] {
+                      return ganns_hnsw_search(h, points, queries_dev, nq, k, l, p, ids_dev,
+                                               dists_dev, stream);
+                    });
 }
 
 int ganns_hnsw_info(const ganns_hnsw* h, int* nlayers, int64_t* layer_n) {

@@ -146,6 +146,19 @@ constexpr int kWideStageRows = 8;   // d > 256: rows per TMA round (4 rounds per
 #ifndef GANNS_SEARCH_ROUNDS
 #define GANNS_SEARCH_ROUNDS 2
 #endif
+// GANNS_LATE_FENCE: the segment form's TMA rounds are issued without a proxy
+// fence (the stage's earlier generic READS are complete: their values were
+// consumed before the issue); the only generic WRITES to the stage (T, by the
+// merge) are followed by fence.proxy.async right after the merge.  Keeps the
+// fence's MEMBAR off the gather's issue path.
+#ifndef GANNS_LATE_FENCE
+#define GANNS_LATE_FENCE 1
+#endif
+// GANNS_SKIP_LB: an exploration none of whose neighbours is below N's l-th key
+// skips the lazy check's binary searches (nothing can enter N)
+#ifndef GANNS_SKIP_LB
+#define GANNS_SKIP_LB 1
+#endif
 #ifndef GANNS_PREFETCH_R2
 #define GANNS_PREFETCH_R2 0
 #endif
@@ -395,7 +408,9 @@ __device__ __forceinline__ float tma_dot(const GraphView& g, const float4 (&qv)[
     const unsigned vm = __ballot_sync(kFull, issuer);
     if (vm) {
       __syncwarp();
-      fence_proxy_async_smem();   // earlier generic reads of the stage precede the async writes
+#if !GANNS_LATE_FENCE
+      fence_proxy_async_smem();   // earlier generic accesses of the stage precede the async writes
+#endif
       if (lane == 0)
         mbar_arrive_expect_tx(ws.mbar, uint32_t(__popc(vm)) * (g4 ? 4u : 1u) * rowbytes);
       __syncwarp();
@@ -674,6 +689,18 @@ __device__ int warp_search_with(const GraphView& g, DIST& dist, int32_t entry, i
     // (4) lazy check (R-C1): drop entries already in N; entries that
     // cannot enter N (>= its l-th key while N is full) are dropped as well.
     const uint64_t worst = cnt == l ? unflag(sN[l - 1]) : kKeyInf;
+#if GANNS_SKIP_LB
+    if (cnt == l) {
+      unsigned below = 0;
+#pragma unroll
+      for (int t = 0; t < TPL; ++t) below |= __ballot_sync(kFull, u[t] >= 0 && key[t] < worst);
+      if (below == 0) {
+        hint = found + 1;
+        __syncwarp();
+        continue;
+      }
+    }
+#endif
     bool cand[TPL];
     int rN[TPL];
     unsigned cb[TPL];
@@ -767,6 +794,9 @@ __device__ int warp_search_with(const GraphView& g, DIST& dist, int32_t entry, i
         if (lane == 0) sBM[c] = 0u;
         __syncwarp();
       }
+#if GANNS_LATE_FENCE
+      fence_proxy_async_smem();   // T's generic writes (in the stage) precede the next TMA writes
+#endif
       hint = pmin < found + 1 ? pmin : found + 1;
     } else {
       hint = found + 1;

@@ -142,6 +142,34 @@ def test_search_deterministic_and_host_path(c1):
     assert (hi.numpy() == a[0]).all() and (hd.numpy() == a[1]).all()
 
 
+def test_search_host_async_two_streams(c1):
+    """ganns_search_host_async: consecutive batches alternating over two streams
+    (the bench's pipeline) give the oracle's results, bit-exact, for every batch."""
+    X, Q, nbr = c1
+    graph = g.from_adjacency(nbr, X.shape[1])
+    Xd = cu(X)
+    k, l, nq = 10, 64, 25
+    batches = [torch.from_numpy(np.ascontiguousarray(Q[i * nq:(i + 1) * nq])).pin_memory()
+               for i in range(len(Q) // nq)]
+    streams = [torch.cuda.Stream(), torch.cuda.Stream()]
+    outs = []
+    for i, qh in enumerate(batches):
+        scratch = (torch.empty((nq, X.shape[1]), dtype=torch.float32, device=DEV),
+                   torch.empty((nq, k), dtype=torch.int32, device=DEV),
+                   torch.empty((nq, k), dtype=torch.float32, device=DEV))
+        hout = (torch.empty((nq, k), dtype=torch.int32).pin_memory(),
+                torch.empty((nq, k), dtype=torch.float32).pin_memory())
+        g.search_host_async(graph, Xd, qh, k, l, scratch, hout, stream=streams[i % 2])
+        outs.append((scratch, hout))
+    torch.cuda.synchronize()
+    oi, od = oracle.search(nbr, X, Q[:nq * len(batches)], k, l, threads=8)
+    for i, (_, (hi, hd)) in enumerate(outs):
+        assert (hi.numpy() == oi[i * nq:(i + 1) * nq]).all()
+        assert (hd.numpy() == od[i * nq:(i + 1) * nq]).all()
+    with pytest.raises(TypeError):   # queries must be pinned host memory
+        g.search_host_async(graph, Xd, torch.from_numpy(Q[:nq]), k, l, outs[0][0], outs[0][1])
+
+
 def test_abi_errors(c1):
     X, Q, nbr = c1
     graph = g.from_adjacency(nbr, X.shape[1])

@@ -18,6 +18,9 @@ ap.add_argument("--l-build", type=int, default=0)
 ap.add_argument("--group", type=int, default=0)
 ap.add_argument("--reps", type=int, default=5)
 ap.add_argument("--nq-mult", default="1", help="comma list: time batches of m x nq queries")
+ap.add_argument("--overlap", type=int, default=0, help="also time this many back-to-back "
+                "batches on one stream and alternating over 2 and 3 streams (no flush between)")
+ap.add_argument("--nqs", default="", help="comma list: also time the first m queries alone")
 ap.add_argument("--orders", default="", help="comma list of pivot counts P: also time the batch "
                 "reordered by each query's nearest of P evenly spaced points (locality experiment)")
 a = ap.parse_args()
@@ -60,6 +63,43 @@ for l in [int(x) for x in a.ls.split(",")]:
             tm.append(e0.elapsed_time(e1) / 1e3)
         tmm = sorted(tm)[len(tm) // 2]
         print(json.dumps({"l": l, "nq": len(Qm), "ms": round(tmm * 1e3, 3), "qps": round(len(Qm) / tmm)}))
+    for m in [int(x) for x in a.nqs.split(",") if x]:
+        Qm = Q[:m].contiguous()
+        tm = []
+        for _ in range(a.reps):
+            flush.zero_()
+            e0, e1 = torch.cuda.Event(True), torch.cuda.Event(True)
+            e0.record()
+            g.search(graph, X, Qm, cfg.k, l)
+            e1.record()
+            e1.synchronize()
+            tm.append(e0.elapsed_time(e1) / 1e3)
+        tmm = sorted(tm)[len(tm) // 2]
+        print(json.dumps({"l": l, "nq": m, "ms": round(tmm * 1e3, 3), "qps": round(m / tmm)}))
+    if a.overlap:
+        outs = [(torch.empty_like(ids), torch.empty(ids.shape, dtype=torch.float32, device="cuda"))
+                for _ in range(a.overlap)]
+        for ns in (1, 2, 3):
+            strs = [torch.cuda.Stream() for _ in range(ns)]
+            tt = []
+            for _ in range(a.reps):
+                flush.zero_()
+                e0, e1 = torch.cuda.Event(True), torch.cuda.Event(True)
+                e0.record()
+                for s_ in strs:
+                    s_.wait_event(e0)
+                for b in range(a.overlap):
+                    g.search(graph, X, Q, cfg.k, l, out=outs[b], stream=strs[b % ns])
+                for s_ in strs:
+                    ev = torch.cuda.Event()
+                    ev.record(s_)
+                    torch.cuda.current_stream().wait_event(ev)
+                e1.record()
+                e1.synchronize()
+                tt.append(e0.elapsed_time(e1) / 1e3)
+            tm_ = sorted(tt)[len(tt) // 2]
+            print(json.dumps({"l": l, "batches": a.overlap, "streams": ns, "ms_per_batch": round(tm_ / a.overlap * 1e3, 3),
+                              "qps": round(a.overlap * len(Q) / tm_)}))
     for P in [int(x) for x in a.orders.split(",") if x]:
         piv = X[:: max(1, len(X) // P)][:P]
         lab = torch.cdist(Q, piv).argmin(1)
