@@ -28,7 +28,7 @@ constexpr int kWarpsPerBlock = 4;   // warps per CTA of the small helper kernels
 constexpr int kSearchWarps = GANNS_SEARCH_WARPS;   // warps (= concurrent queries) per CTA
 constexpr int kSearchPool = GANNS_SEARCH_POOL;     // shared stage buffers per CTA (0: one per warp)
 #ifndef GANNS_MIN_BLOCKS
-#define GANNS_MIN_BLOCKS 12
+#define GANNS_MIN_BLOCKS (24 / GANNS_SEARCH_WARPS)
 #endif
 constexpr int kMinBlocksPerSM = GANNS_MIN_BLOCKS; // register budget: <= 85 regs/thread (24 warps per SM);
                                     // the TMA stage (8 KB/warp at d=128) allows ~22 warps

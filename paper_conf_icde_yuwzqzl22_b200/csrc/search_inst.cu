@@ -18,7 +18,7 @@ namespace ganns {
 #endif
 // 2 warps per CTA, 2-round form: a warp whose sibling has left takes over both
 // stages (1 round per exploration) -- shortens the drain of a batch
-constexpr bool kPairStages = GANNS_PAIR_STAGES != 0 && GANNS_SEARCH_WARPS == 2 &&
+constexpr bool kPairStages = GANNS_PAIR_STAGES != 0 && GANNS_SEARCH_WARPS % 2 == 0 &&
                              GANNS_SEARCH_ROUNDS == 2 && GANNS_SEARCH_POOL == 0;
 
 // Persistent: every warp pulls queries from a per-launch ticket counter until
@@ -44,15 +44,16 @@ search_kernel(GraphView g, const float* __restrict__ Q, int64_t nq, int k, int l
     }
     __syncthreads();
   } else if (kPairStages && uses_tma(NV4)) {
-    // [stage 0][stage 1][warp 0: N/mbar/bitmap][warp 1: ...][flag]; each stage
-    // region also holds its warp's T (ganns_dev.cuh: t_bytes)
+    // [stage 0 .. W-1][warp 0: N/mbar/bitmap .. warp W-1][one flag per warp pair];
+    // each stage region also holds its warp's T (ganns_dev.cuh: t_bytes); warps
+    // 2p and 2p+1 are partners with contiguous stages
     const size_t sb = stage_region_bytes(NV4, g.d4, kSearchStageRounds, TPL);
     const size_t rb = warp_tail_bytes(l);
     ws = carve_warp_smem(smem + size_t(w) * sb, l, TPL, NV4, g.d4, kSearchStageRounds);
-    carve_warp_tail(ws, smem + 2 * sb + size_t(w) * rb, l);
-    ws.pair_stage = reinterpret_cast<float4*>(smem);
-    ws.pair_flag = reinterpret_cast<volatile int*>(smem + 2 * sb + 2 * rb);
-    if (threadIdx.x == 0) *ws.pair_flag = 0;
+    carve_warp_tail(ws, smem + kSearchWarps * sb + size_t(w) * rb, l);
+    ws.pair_stage = reinterpret_cast<float4*>(smem + size_t(w & ~1) * sb);
+    ws.pair_flag = reinterpret_cast<volatile int*>(smem + kSearchWarps * (sb + rb)) + (w >> 1);
+    if (lane == 0 && (w & 1) == 0) *ws.pair_flag = 0;
     if (lane == 0) mbar_init(ws.mbar, 1);
     __syncthreads();
   } else {
@@ -136,8 +137,9 @@ static cudaError_t launch_t(const SearchLaunch& a, cudaStream_t s) {
                     ? pooled_cta_bytes(a.l, TPL, NV4, a.d / 4, kSearchStageRounds, kSearchWarps,
                                        kSearchPool)
                 : kPairStages && uses_tma(NV4)
-                    ? 2 * (stage_region_bytes(NV4, a.d / 4, kSearchStageRounds, TPL) +
-                           warp_tail_bytes(a.l)) + 16
+                    ? kSearchWarps * (stage_region_bytes(NV4, a.d / 4, kSearchStageRounds, TPL) +
+                                      warp_tail_bytes(a.l)) +
+                          ((kSearchWarps / 2 * 4 + 15) & ~15)
                     : size_t(kSearchWarps) *
                           warp_smem_bytes(a.l, TPL, NV4, a.d / 4, kSearchStageRounds, wrows);
   if (smem > 227 * 1024) return cudaErrorInvalidValue;
