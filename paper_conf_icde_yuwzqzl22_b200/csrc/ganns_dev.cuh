@@ -107,6 +107,16 @@ __device__ __forceinline__ float4 lds128_ordered(const float4* p) {
                : "=f"(r.x), "=f"(r.y), "=f"(r.z), "=f"(r.w) : "r"(smem_u32(p)));
   return r;
 }
+// stage hand-over of a warp pair (named barrier `id`, the pair's 64 threads)
+// (non-.aligned forms: the two warps reach the barrier through different instructions)
+__device__ __forceinline__ void pair_bar_arrive(int id) {
+  __syncwarp();
+  asm volatile("barrier.arrive %0, 64;" ::"r"(id) : "memory");
+}
+__device__ __forceinline__ void pair_bar_sync(int id) {
+  __syncwarp();
+  asm volatile("barrier.sync %0, 64;" ::"r"(id) : "memory");
+}
 __device__ __forceinline__ void fence_proxy_async_smem() {
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
 }
@@ -215,6 +225,7 @@ struct WarpSmem {
   // round trip per exploration for the last queries of a batch
   float4* pair_stage;
   volatile int* pair_flag;
+  int pair_bar;   // named barrier of the pair (64 threads): leaver arrives, taker syncs
 };
 // Per-CTA layout of the pooled search kernel: [pool stages][per-warp N/T/bitmap][pool meta]
 __host__ __device__ constexpr size_t pooled_warp_bytes(int l, int tpl) {
@@ -595,6 +606,10 @@ struct WarpDist {
         int f = 0;
         if (lane == 0) f = atomicAdd(const_cast<int*>(ws.pair_flag), 0);   // atomic: orders the handover
         if (__shfl_sync(kFull, f, 0) != 0) {
+          // the sibling has left: its bar.arrive (after its last writes to its
+          // stage, which held its T) pairs with this bar.sync -- a CTA-level
+          // happens-before edge for the stage hand-over
+          pair_bar_sync(ws.pair_bar);
           ws.rounds = 1;
           ws.stage = ws.pair_stage;
         }

@@ -53,6 +53,7 @@ search_kernel(GraphView g, const float* __restrict__ Q, int64_t nq, int k, int l
     carve_warp_tail(ws, smem + kSearchWarps * sb + size_t(w) * rb, l);
     ws.pair_stage = reinterpret_cast<float4*>(smem + size_t(w & ~1) * sb);
     ws.pair_flag = reinterpret_cast<volatile int*>(smem + kSearchWarps * (sb + rb)) + (w >> 1);
+    ws.pair_bar = 1 + (w >> 1);
     if (lane == 0 && (w & 1) == 0) *ws.pair_flag = 0;
     if (lane == 0) mbar_init(ws.mbar, 1);
     __syncthreads();
@@ -70,7 +71,16 @@ search_kernel(GraphView g, const float* __restrict__ Q, int64_t nq, int k, int l
   const int64_t q = __shfl_sync(kFull, qt, 0);
   if (q >= nq) {
     // this warp's stage is idle from now on: the sibling may take it over
-    if (ws.pair_flag != nullptr && lane == 0) atomicExch(const_cast<int*>(ws.pair_flag), 1);
+    if (ws.pair_flag != nullptr && ws.rounds == 2) {
+      // hand the stage to the sibling: this warp's last stage writes (its T) are
+      // ordered before the sibling's TMA by the pair barrier (arrive here, sync
+      // there when it takes the stage, or arrive when it leaves as well)
+      fence_proxy_async_smem();
+      __threadfence_block();
+      if (lane == 0) atomicExch(const_cast<int*>(ws.pair_flag), 1);
+      __syncwarp();
+      pair_bar_arrive(ws.pair_bar);
+    }
     break;
   }
   SearchStats st;
