@@ -99,11 +99,11 @@ class ClockSampler:
         self.samples.append((sm, rs))
 
     def _run(self):
-        while not self.stop.is_set():
+        fails = 0
+        while not self.stop.is_set() and fails < 100:
             n = len(self.samples)
             self.sample_now()
-            if len(self.samples) == n:
-                break
+            fails += len(self.samples) == n   # a failed NVML read: retry, give up after 100
             time.sleep(0.002)
 
     def __enter__(self):

@@ -204,7 +204,8 @@ GANNS_API int ganns_build_hnsw(const float *points, int64_t n, int d, int metric
                                void *stream, ganns_hnsw **out);
 
 /* ganns_hnsw_search -- ganns_search_ex on the HNSW index; p->entry is ignored
- * (each query enters layer 0 where its descent ends).  Launches two kernels. */
+ * (each query enters layer 0 where its descent ends).  d <= 256: one kernel (the
+ * descent runs inside K1); d > 256: an entry kernel, then K1. */
 GANNS_API int ganns_hnsw_search(const ganns_hnsw *h, const float *points, const float *queries,
                                 int64_t nq, int k, int l, const ganns_search_params *p,
                                 int32_t *out_ids, float *out_dists, void *stream);

@@ -626,6 +626,26 @@ int ganns_hnsw_search(const ganns_hnsw* h, const float* points, const float* que
     return rc;
   if (nq == 0) return GANNS_OK;
   cudaStream_t s = static_cast<cudaStream_t>(stream);
+  const ganns_graph* g = h->base;
+  if (h->nlayers > 1 && nv4_for(h->d) <= 2) {
+    // d <= 256: the descent runs inside K1, one launch (search_inst.cu: HnswUpper)
+    UpperLayersHost up;
+    up.top = h->nlayers - 1;
+    for (int j = 1; j < h->nlayers; ++j) {
+      up.nbr[j] = h->upper[j];
+      up.n[j] = h->layer_n[j];
+    }
+    int32_t* tk = ticket_slot();
+    if (!tk) return fail(GANNS_ENOMEM, "ticket allocation failed");
+    SearchLaunch a{g->nbr, points, g->n, g->d, g->d_max, g->metric, queries, nq, k, l, e, entry,
+                   out_ids, out_dists, p ? p->stats : nullptr, tk};
+    a.upper = &up;
+    a.Xp = h->Xp;
+    a.np = h->layer_n[1];
+    a.perm = h->perm;
+    cudaError_t err = launch_search(a, s);
+    return err == cudaSuccess ? GANNS_OK : cuda_fail(err, "hnsw search");
+  }
   int32_t* entries = nullptr;
   if (cudaMallocAsync(&entries, sizeof(int32_t) * nq, s) != cudaSuccess)
     return fail(GANNS_ENOMEM, "cudaMallocAsync(entries)");
@@ -658,7 +678,6 @@ int ganns_hnsw_search(const ganns_hnsw* h, const float* points, const float* que
   }
   int32_t* tk = ticket_slot();
   if (!tk) return fail(GANNS_ENOMEM, "ticket allocation failed");
-  const ganns_graph* g = h->base;
   SearchLaunch a{g->nbr, points, g->n, g->d, g->d_max, g->metric, queries, nq, k, l, e, entry,
                  out_ids, out_dists, p ? p->stats : nullptr, tk};
   a.entries = entries;

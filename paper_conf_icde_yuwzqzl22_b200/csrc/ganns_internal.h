@@ -68,6 +68,12 @@ struct SearchLaunch {
   uint32_t* stats;
   int32_t* ticket;      // device scratch counter for the persistent scheduler
   const int32_t* entries = nullptr;   // per-query entry vertices (HNSW), nullable
+  // HNSW with the descent fused into K1 (d <= 256): upper layers over the permuted
+  // rows Xp [np][d]; a query enters layer 0 at perm[vertex its descent reaches]
+  const UpperLayersHost* upper = nullptr;
+  const float* Xp = nullptr;
+  int64_t np = 0;
+  const int32_t* perm = nullptr;
 };
 // HNSW: per-query layer-0 entry = perm[greedy descent through the upper layers]
 struct EntryLaunch {

@@ -23,13 +23,24 @@ constexpr bool kPairStages = GANNS_PAIR_STAGES != 0 && GANNS_SEARCH_WARPS % 2 ==
 
 // Persistent: every warp pulls queries from a per-launch ticket counter until
 // the batch is exhausted, so the last wave is balanced at query granularity.
-template <int NV4, int TPL, bool L2>
+// HNSW (Section IV-D): each query first descends the upper layers
+// greedily (the GANNS search with l = e = 1 per layer, over the permuted rows Xp)
+// in the same warp, then searches layer 0 from perm[vertex reached] -- no separate
+// entry kernel, and the descent's latency hides behind the other warps' searches.
+struct HnswUpper {
+  UpperLayers U;
+  const float* Xp;
+  int64_t np;
+  const int32_t* perm;
+};
+template <int NV4, int TPL, bool L2, bool HNSW>
 __global__ void __launch_bounds__(kSearchWarps * 32, kMinBlocksPerSM)
 search_kernel(GraphView g, const float* __restrict__ Q, int64_t nq, int k, int l, int e,
               int32_t entry, int32_t* __restrict__ out_ids, float* __restrict__ out_dists,
               uint32_t* __restrict__ stats, int32_t* __restrict__ ticket,
               const int32_t* __restrict__ entries, int wrows,
-              const __grid_constant__ CUtensorMap tmap) {
+              const __grid_constant__ CUtensorMap tmap, const __grid_constant__ HnswUpper H,
+              const __grid_constant__ CUtensorMap tmap_up) {
   g.tmap = &tmap;
   extern __shared__ __align__(128) uint8_t smem[];
   const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -84,9 +95,16 @@ search_kernel(GraphView g, const float* __restrict__ Q, int64_t nq, int k, int l
     break;
   }
   SearchStats st;
-  const int32_t ent = entries != nullptr ? entries[q] : entry;   // HNSW: per-query entry
-  const int cnt = warp_search<NV4, TPL, L2, false>(g, Q + size_t(q) * (g.d4 * 4), ent, l, e,
-                                                   ws, st);
+  const float* qrow = Q + size_t(q) * (g.d4 * 4);
+  int32_t ent = entries != nullptr ? entries[q] : entry;   // HNSW: per-query entry
+  if constexpr (HNSW) {
+    GraphView gu = g;
+    gu.X = H.Xp;
+    gu.n = H.np;
+    gu.tmap = &tmap_up;
+    ent = H.perm[descend<NV4, TPL, L2>(gu, H.U, 1, qrow, ws)];
+  }
+  const int cnt = warp_search<NV4, TPL, L2, false>(g, qrow, ent, l, e, ws, st);
   // output: the first k of N, (-1, +inf) padded (R-C8)
   for (int i = lane; i < k; i += 32) {
     uint64_t key = i < cnt ? unflag(sN[i]) : kKeyInf;
@@ -119,7 +137,7 @@ static int pick_wide_rows(const SearchLaunch& a, int sms) {
     int per_sm = 0;
     const size_t smem = size_t(kSearchWarps) * warp_smem_bytes(a.l, TPL, NV4, a.d / 4,
                                                                kSearchStageRounds, r);
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, search_kernel<NV4, TPL, L2>,
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, search_kernel<NV4, TPL, L2, false>,
                                                       kSearchWarps * 32, smem) != cudaSuccess)
       return kWideStageRows;
     if (int64_t(per_sm) * sms * kSearchWarps >= a.nq) return r;
@@ -127,9 +145,9 @@ static int pick_wide_rows(const SearchLaunch& a, int sms) {
   return kWideStageRows;
 }
 
-template <int NV4, int TPL, bool L2>
+template <int NV4, int TPL, bool L2, bool HNSW = false>
 static cudaError_t launch_t(const SearchLaunch& a, cudaStream_t s) {
-  auto kern = search_kernel<NV4, TPL, L2>;
+  auto kern = search_kernel<NV4, TPL, L2, HNSW>;
   static bool attr_done = false;   // per instantiation
   if (!attr_done) {
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -165,6 +183,22 @@ static cudaError_t launch_t(const SearchLaunch& a, cudaStream_t s) {
   CUtensorMap tmap;
   cudaError_t err = uses_tma(NV4) ? encode_row_tmap(a.X, a.n, a.d, &tmap) : zero_tmap(&tmap);
   if (err != cudaSuccess) return err;
+  HnswUpper H{};
+  CUtensorMap tmap_up;
+  err = zero_tmap(&tmap_up);
+  if (err != cudaSuccess) return err;
+  if constexpr (HNSW) {
+    H.U.top = a.upper->top;
+    for (int j = 0; j < kMaxLayers; ++j) {
+      H.U.nbr[j] = a.upper->nbr[j];
+      H.U.n[j] = a.upper->n[j];
+    }
+    H.Xp = a.Xp;
+    H.np = a.np;
+    H.perm = a.perm;
+    err = encode_row_tmap(a.Xp, a.np, a.d, &tmap_up);
+    if (err != cudaSuccess) return err;
+  }
   err = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kSearchWarps * 32, smem);
   if (err != cudaSuccess) return err;
   int64_t blocks = (a.nq + kSearchWarps - 1) / kSearchWarps;
@@ -174,7 +208,7 @@ static cudaError_t launch_t(const SearchLaunch& a, cudaStream_t s) {
   if (err != cudaSuccess) return err;
   kern<<<dim3(unsigned(blocks)), kSearchWarps * 32, smem, s>>>(
       g, a.Q, a.nq, a.k, a.l, a.e, a.entry, a.out_ids, a.out_dists, a.stats, a.ticket, a.entries,
-      wrows, tmap);
+      wrows, tmap, H, tmap_up);
   count_launch();
   return cudaGetLastError();
 }
@@ -254,6 +288,10 @@ static cudaError_t launch_m(const SearchLaunch& a, cudaStream_t s) {
 #ifdef GANNS_DEV_ONE
   return launch_t<NV4, TPL, true>(a, s);
 #endif
+  if constexpr (uses_tma(NV4))
+    if (a.upper != nullptr && a.upper->top > 0)
+      return a.metric == 0 ? launch_t<NV4, TPL, true, true>(a, s)
+                           : launch_t<NV4, TPL, false, true>(a, s);
   return a.metric == 0 ? launch_t<NV4, TPL, true>(a, s) : launch_t<NV4, TPL, false>(a, s);
 }
 template <int NV4>
