@@ -5,7 +5,8 @@
 // One warp owns one query (the paper's "thread block per query" with n_t = 32
 // threads, R-C20).  Per query the warp keeps, in shared memory:
 //   sN  : candidate array N, up to l packed keys (lazy update), ascending
-//   sT  : the surviving visiting entries T, compacted in sorted order
+//   sT  : the surviving visiting entries T, compacted in sorted order;
+//         it lives inside the TMA stage (idle during the merge)
 //   sBM : a bitmap of the positions of N that T entries land on in the merge
 // A key is (orderable fp32 distance << 32) | id; bit 31 of the id word is the
 // "explored" flag, so the flag travels with its entry through the merge.
@@ -16,9 +17,10 @@
 //   (1) candidate locating  -- __ballot_sync / __ffs over 32-entry chunks of N
 //       from a "first possibly unexplored" hint
 //   (2) neighbourhood exploration -- one coalesced load of the adjacency row
-//   (3) bulk distance -- all d_max rows gathered with 128-bit read-only loads,
-//       B rows in flight per lane; partial dot products reduced by a transposing
-//       butterfly so lane j ends with delta(q, T[j])
+//   (3) bulk distance -- the neighbour rows gathered by TMA (tile::gather4, or
+//       1-D bulk copies) into the warp's shared-memory stage, all rows of a round
+//       in flight on one mbarrier; partial sums reduced by a transposing butterfly
+//       so lane j ends with delta(q, T[j])
 //   (4) lazy check -- entries that cannot enter N (>= its l-th key when full)
 //       are skipped; the rest binary-search N; equal key => duplicate, dropped
 //       (R-C1).  The probe gives rank_N(t) for free.

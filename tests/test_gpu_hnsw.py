@@ -73,3 +73,38 @@ def test_hnsw_c2_recall_beats_or_matches_nsw():
     rh, rn = oracle.recall(hi.cpu().numpy(), gt), oracle.recall(ni.cpu().numpy(), gt)
     assert rh >= rn - 0.005, (rh, rn)
     assert hs[:, 0].float().mean() <= ns[:, 0].float().mean() + 1.0
+
+
+def test_hnsw_wide_rows_entry_kernel_path():
+    """d > 256: the search takes the separate entry-kernel path (the descent is fused
+    into K1 only for d <= 256); bit-exact vs the oracle as well."""
+    n, d = 1500, 384
+    X = syn.random_int_points(n, d, 0, 15, 11)
+    Q = syn.random_int_points(60, d, 0, 15, 12)
+    levels = syn.hnsw_levels(n, 8, 5)
+    ref = oracle.hnsw_build(X, levels, 8, 16, 128, l_build=32)
+    idx = g.build_hnsw(cu(X), levels, degree=16, l_build=32, group_size=128)
+    assert (idx.layer(0) == ref["layer0"]).all()
+    ids, dists, st = g.hnsw_search(idx, cu(X), cu(Q), 10, 40, stats=True)
+    oi, od, _, ost = oracle.hnsw_search(ref, X, Q, 10, 40, stats=True)
+    assert (ids.cpu().numpy() == oi).all() and (dists.cpu().numpy() == od).all()
+    assert (st.cpu().numpy()[:, 0] == ost[:, 0]).all()
+
+
+def test_hnsw_search_host_async():
+    """ganns_hnsw_search_host_async (H2D, search, D2H on a stream) == hnsw_search."""
+    cfg = syn.with_size(syn.CONFIGS["C1"], n=3000, nq=64)
+    X, Q = syn.points(cfg), syn.queries(cfg)
+    levels = syn.hnsw_levels(3000, 8, 2)
+    idx = g.build_hnsw(cu(X), levels, degree=16, l_build=32, group_size=128)
+    Xd = cu(X)
+    ids, dists = g.hnsw_search(idx, Xd, cu(Q), 10, 48)
+    scratch = (torch.empty((64, X.shape[1]), dtype=torch.float32, device=DEV),
+               torch.empty((64, 10), dtype=torch.int32, device=DEV),
+               torch.empty((64, 10), dtype=torch.float32, device=DEV))
+    hout = (torch.empty((64, 10), dtype=torch.int32).pin_memory(),
+            torch.empty((64, 10), dtype=torch.float32).pin_memory())
+    s = torch.cuda.Stream()
+    g.search_host_async(idx, Xd, torch.from_numpy(Q).pin_memory(), 10, 48, scratch, hout, stream=s)
+    s.synchronize()
+    assert (hout[0] == ids.cpu()).all() and (hout[1] == dists.cpu()).all()
