@@ -112,6 +112,24 @@ def _stream(stream) -> ct.c_void_p:
     return ct.c_void_p(stream.cuda_stream)
 
 
+def _check_buf(t, shape, dtype, cuda: bool, name: str):
+    """Output / scratch buffers are written by the library through raw pointers:
+    refuse anything that is not exactly the expected contiguous layout."""
+    if not (isinstance(t, torch.Tensor) and tuple(t.shape) == tuple(shape) and t.dtype == dtype
+            and t.is_cuda == cuda and t.is_contiguous()):
+        where = "CUDA" if cuda else "host"
+        raise TypeError(f"{name} must be a contiguous {where} {dtype} tensor of shape {tuple(shape)}")
+
+
+def _check_out(out, nq: int, k: int, device):
+    ids, dists = out
+    _check_buf(ids, (nq, k), torch.int32, True, "out[0] (ids)")
+    _check_buf(dists, (nq, k), torch.float32, True, "out[1] (dists)")
+    if ids.device != device or dists.device != device:
+        raise TypeError("out tensors must be on the queries' device")
+    return ids, dists
+
+
 def _dev_f32(t: torch.Tensor, name: str) -> torch.Tensor:
     if not (isinstance(t, torch.Tensor) and t.is_cuda and t.dtype == torch.float32 and t.dim() == 2):
         raise TypeError(f"{name} must be a 2-D float32 CUDA tensor")
@@ -208,7 +226,7 @@ def search(graph: Graph, points: torch.Tensor, queries: torch.Tensor, k: int, l:
         ids = torch.empty((nq, k), dtype=torch.int32, device=queries.device)
         dists = torch.empty((nq, k), dtype=torch.float32, device=queries.device)
     else:
-        ids, dists = out
+        ids, dists = _check_out(out, nq, k, queries.device)
     st = torch.empty((nq, 3), dtype=torch.int32, device=queries.device) if stats else None
     p = _SearchParams(e, entry, ct.c_void_p(st.data_ptr()) if stats else None)
     with torch.cuda.device(queries.device):
@@ -233,6 +251,8 @@ def search_host(graph: Graph, points: torch.Tensor, queries: torch.Tensor, k: in
         dists = torch.empty((nq, k), dtype=torch.float32, pin_memory=True)
     else:
         ids, dists = out
+        _check_buf(ids, (nq, k), torch.int32, False, "out[0] (ids)")
+        _check_buf(dists, (nq, k), torch.float32, False, "out[1] (dists)")
     p = _SearchParams(e, entry, None)
     with torch.cuda.device(points.device):
         _check(_lib.ganns_search_host(graph.handle, ct.c_void_p(points.data_ptr()),
@@ -258,6 +278,14 @@ def search_host_async(index, points: torch.Tensor, queries_host: torch.Tensor, k
         raise TypeError("out_host must be pinned CPU tensors")
     qd, ids_d, dists_d = scratch
     nq = queries_host.shape[0]
+    if queries_host.dim() != 2 or not queries_host.is_contiguous():
+        raise TypeError("queries_host must be a contiguous 2-D tensor")
+    d = queries_host.shape[1]
+    _check_buf(qd, (nq, d), torch.float32, True, "scratch[0] (queries)")
+    _check_buf(ids_d, (nq, k), torch.int32, True, "scratch[1] (ids)")
+    _check_buf(dists_d, (nq, k), torch.float32, True, "scratch[2] (dists)")
+    _check_buf(ids_h, (nq, k), torch.int32, False, "out_host[0] (ids)")
+    _check_buf(dists_h, (nq, k), torch.float32, False, "out_host[1] (dists)")
     p = _SearchParams(e, 0, None)
     fn = _lib.ganns_hnsw_search_host_async if isinstance(index, Hnsw) else _lib.ganns_search_host_async
     with torch.cuda.device(points.device):
@@ -362,7 +390,7 @@ def hnsw_search(index: Hnsw, points: torch.Tensor, queries: torch.Tensor, k: int
         ids = torch.empty((nq, k), dtype=torch.int32, device=queries.device)
         dists = torch.empty((nq, k), dtype=torch.float32, device=queries.device)
     else:
-        ids, dists = out
+        ids, dists = _check_out(out, nq, k, queries.device)
     st = torch.empty((nq, 3), dtype=torch.int32, device=queries.device) if stats else None
     p = _SearchParams(e, 0, ct.c_void_p(st.data_ptr()) if stats else None)
     with torch.cuda.device(queries.device):

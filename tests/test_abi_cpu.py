@@ -49,3 +49,18 @@ def test_last_error_without_gpu_calls():
     lib.ganns_graph_info.restype = ctypes.c_int
     assert lib.ganns_graph_info(None, None, None, None, None) == -1   # EINVAL on NULL graph
     assert b"NULL" in lib.ganns_last_error()
+
+
+def test_binding_refuses_mis_shaped_output_buffers():
+    """Buffers the library writes through raw pointers are checked in the binding."""
+    import pytest
+    import torch
+    import paper_conf_icde_yuwzqzl22_b200 as g
+    ok = torch.empty((4, 10), dtype=torch.int32)
+    g._check_buf(ok, (4, 10), torch.int32, False, "x")
+    for bad in (torch.empty((4, 9), dtype=torch.int32), torch.empty((4, 10), dtype=torch.int64),
+                torch.empty((10, 4), dtype=torch.int32).t()):
+        with pytest.raises(TypeError):
+            g._check_buf(bad, (4, 10), torch.int32, False, "x")
+    with pytest.raises(TypeError):   # host tensor where a CUDA one is required
+        g._check_buf(ok, (4, 10), torch.int32, True, "x")
