@@ -37,7 +37,8 @@ sys.path.insert(0, ROOT)
 
 import ganns_synth as syn  # noqa: E402
 
-L_SWEEP = [32, 40, 48, 56, 64, 80, 96, 112, 128, 160, 192, 256, 320, 384, 512]
+L_SWEEP = [32, 40, 48, 56, 64, 72, 80, 88, 96, 104, 112, 120, 128, 144, 160, 192, 224, 256, 288,
+           320, 352, 384, 448, 512]
 
 
 def parse():
@@ -331,7 +332,8 @@ def select_operating_point(torch, index, Qd, gt, k, target, timer):
 
     for l in L_SWEEP:
         best_r = 0.0
-        es = {l, max(k, int(round(0.85 * l))), max(k, int(round(0.7 * l)))}
+        es = {l, max(k, int(round(0.92 * l))), max(k, int(round(0.85 * l))),
+              max(k, int(round(0.7 * l)))}
         if len(feasible) >= 6:
             es = {l}   # only looking for the 0.99 operating point now
         for e in sorted(es, reverse=True):
