@@ -51,6 +51,9 @@ def parse():
     ap.add_argument("--target", type=float, default=0.95)
     ap.add_argument("--l-build", type=int, default=128,
                     help="candidate-list length of the build searches (P:222: 32/64/128)")
+    ap.add_argument("--l-local", type=int, default=64,
+                    help="list length of the Phase-1 (local graph) build searches, <= l_build "
+                         "(R-C13; 0 = l_build); not used by the HNSW config")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
     ap.add_argument("--json-out", default=None)
@@ -195,7 +198,7 @@ class BenchIndex:
     for the GloVe-shaped config (BASELINE configs[3]) -- the HNSW-style graph of
     Section IV-D with seeded levels."""
 
-    def __init__(self, g, cfg, Xd, l_build):
+    def __init__(self, g, cfg, Xd, l_build, l_local=0):
         self.g, self.cfg, self.Xd = g, cfg, Xd
         self.hnsw = cfg.name == "C4"
         if self.hnsw:
@@ -206,7 +209,8 @@ class BenchIndex:
             self.build_stats = self.idx.build_stats
         else:
             self.idx = None
-            self.graph = g.build(Xd, metric=cfg.metric, degree=cfg.degree, l_build=l_build)
+            self.graph = g.build(Xd, metric=cfg.metric, degree=cfg.degree, l_build=l_build,
+                                 l_local=min(l_local, l_build))
             self.build_stats = self.graph.build_stats
         self.kind = "HNSW-style (Section IV-D)" if self.hnsw else "NSW (Algorithm 2)"
 
@@ -387,7 +391,7 @@ def run_ours(args):
 
     # ---- GGraphCon build (timed wall clock on device-resident points)
     t0 = time.perf_counter()
-    index = BenchIndex(g, cfg, Xd, args.l_build)
+    index = BenchIndex(g, cfg, Xd, args.l_build, args.l_local)
     torch.cuda.synchronize()
     build_s = time.perf_counter() - t0
     b_iters, b_comps, b_searches, b_rounds = index.build_stats
@@ -493,6 +497,8 @@ def run_ours(args):
                    "parallelism": f"replicated graph, query data-parallel x{world}"},
         "build_seconds": round(build_s, 4),
         "build_params": {"degree": cfg.degree, "d_min": cfg.degree // 2, "l_build": args.l_build,
+                         "l_local": (None if index.hnsw else min(args.l_local, args.l_build) or
+                                     args.l_build),
                          "group_size": "auto"},
         "build": {"iterations": b_iters, "distance_computations": b_comps,
                   "searches": b_searches, "rounds": b_rounds,
@@ -515,7 +521,8 @@ def run_ours(args):
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         line["cpu_baseline"] = cpu_baseline(index, X, Q, k, l_star, e_star, args.cpu_seconds)
         if not index.hnsw:
-            line["cpu_build_baseline"] = cpu_build_baseline(torch, g, cfg, X, args.l_build)
+            line["cpu_build_baseline"] = cpu_build_baseline(torch, g, cfg, X, args.l_build,
+                                                            min(args.l_local, args.l_build))
     if rank == 0:
         s = json.dumps(line)
         print(s, flush=True)
@@ -560,7 +567,8 @@ def run_sharded(args):
         Xs = torch.from_numpy(syn.points(cfg, s * per, (s + 1) * per)).to(dev)
         torch.cuda.synchronize()
         t0 = time.perf_counter()
-        gr = g.build(Xs, metric=cfg.metric, degree=cfg.degree, l_build=args.l_build)
+        gr = g.build(Xs, metric=cfg.metric, degree=cfg.degree, l_build=args.l_build,
+                     l_local=min(args.l_local, args.l_build))
         torch.cuda.synchronize()
         build_s = max(build_s, time.perf_counter() - t0)
         gi_s, gd_s = ground_truth(torch, Xs, Qd[:nsub], k, cfg.metric, with_dist=True)
@@ -764,7 +772,7 @@ def cpu_baseline(index, X, Q, k, l, e, seconds):
             "sample": f"first {m2} of the {len(Q)} queries, same graph, l={l}, e={e}, {dt:.1f} s"}
 
 
-def cpu_build_baseline(torch, g, cfg, X, l_build, m=10000):
+def cpu_build_baseline(torch, g, cfg, X, l_build, l_local=0, m=10000):
     """Algorithm 2 on the first m points: the oracle (plain C, one thread -- the paper's
     CPU baselines are single-threaded) and the GPU build of the same sample with
     the same partition (group size 256 = the auto rule at this size)."""
@@ -772,18 +780,21 @@ def cpu_build_baseline(torch, g, cfg, X, l_build, m=10000):
     Xs = np.ascontiguousarray(X[:m])
     S = 256
     t0 = time.perf_counter()
-    oracle.alg2(Xs, cfg.degree // 2, cfg.degree, S, l_build=l_build, metric=cfg.metric)
+    oracle.alg2(Xs, cfg.degree // 2, cfg.degree, S, l_build=l_build, metric=cfg.metric,
+                l_local=l_local)
     t_cpu = time.perf_counter() - t0
     Xd = torch.from_numpy(Xs).cuda()
-    g.build(Xd, metric=cfg.metric, degree=cfg.degree, l_build=l_build, group_size=S)  # warm
+    g.build(Xd, metric=cfg.metric, degree=cfg.degree, l_build=l_build, group_size=S,
+            l_local=l_local)  # warm
     torch.cuda.synchronize()
     t0 = time.perf_counter()
-    g.build(Xd, metric=cfg.metric, degree=cfg.degree, l_build=l_build, group_size=S)
+    g.build(Xd, metric=cfg.metric, degree=cfg.degree, l_build=l_build, group_size=S,
+            l_local=l_local)
     torch.cuda.synchronize()
     t_gpu = time.perf_counter() - t0
     return {"oracle_s": round(t_cpu, 3), "gpu_s": round(t_gpu, 4), "cores": 1, "kind": "oracle",
             "sample": f"Algorithm 2 on the first {m} points (degree {cfg.degree}, "
-                      f"l_build {l_build}, group size {S})"}
+                      f"l_build {l_build}, l_local {l_local or l_build}, group size {S})"}
 
 
 def run_reference(args):
@@ -803,7 +814,7 @@ def run_reference(args):
     # index set-up (not timed): the graph the GPU arm searches (deterministic) and
     # the same (l, e) operating point, selected the same way
     Xd = torch.from_numpy(X).cuda()
-    index = BenchIndex(g, cfg, Xd, args.l_build)
+    index = BenchIndex(g, cfg, Xd, args.l_build, args.l_local)
     Qd = torch.from_numpy(np.concatenate(Qs)).cuda()
     gt = ground_truth(torch, Xd, Qd, k, cfg.metric)
     Qds = [Qd[b * len(Q):(b + 1) * len(Q)] for b in range(len(Qs))]

@@ -68,6 +68,10 @@ typedef struct {
     int stop_after_phase1; /* != 0: return the union of local graphs (parity hook)         */
     uint64_t *stats;    /* host, nullable, [4]: search iterations, distance computations,
                            searches, rounds -- filled when ganns_build returns             */
+    int l_local;        /* list length of the Phase-1 searches on the local graphs (lines
+                           4-5); 0 -> l_build; else in [d_min, l_build]; their explore
+                           budget is min(e_build, l_local) (R-C13: the paper leaves both
+                           lengths open).  Ignored by ganns_build_hnsw.                    */
 } ganns_build_params;
 
 /* Extra search parameters.  Zero-initialise for defaults. */

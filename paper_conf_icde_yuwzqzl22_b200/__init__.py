@@ -29,7 +29,8 @@ class GannsError(RuntimeError):
 class _BuildParams(ct.Structure):
     _fields_ = [("d_min", ct.c_int), ("l_build", ct.c_int), ("e_build", ct.c_int),
                 ("group_size", ct.c_int64), ("max_rounds", ct.c_int),
-                ("stop_after_phase1", ct.c_int), ("stats", ct.POINTER(ct.c_uint64))]
+                ("stop_after_phase1", ct.c_int), ("stats", ct.POINTER(ct.c_uint64)),
+                ("l_local", ct.c_int)]
 
 
 class _SearchParams(ct.Structure):
@@ -197,14 +198,14 @@ def from_adjacency(nbr: np.ndarray, d: int, metric: str = "l2", device: int = 0)
 
 def build(points: torch.Tensor, metric: str = "l2", degree: int = 32, d_min: int = 0,
           l_build: int = 0, e_build: int = 0, group_size: int = 0, max_rounds: int = 0,
-          stop_after_phase1: bool = False, stream=None) -> Graph:
+          stop_after_phase1: bool = False, l_local: int = 0, stream=None) -> Graph:
     """GGraphCon NSW construction (Algorithm 2).  ``points`` [n, d] float32 CUDA
     (unit rows for metric="cosine").  Returns a Graph; ``graph.build_stats`` =
     (search iterations, distance computations, searches, rounds)."""
     points = _dev_f32(points, "points")
     st = (ct.c_uint64 * 4)()
     p = _BuildParams(d_min, l_build, e_build, group_size, max_rounds, int(stop_after_phase1),
-                     ct.cast(st, ct.POINTER(ct.c_uint64)))
+                     ct.cast(st, ct.POINTER(ct.c_uint64)), l_local)
     h = ct.c_void_p()
     with torch.cuda.device(points.device):
         _check(_lib.ganns_build(ct.c_void_p(points.data_ptr()), points.shape[0], points.shape[1],

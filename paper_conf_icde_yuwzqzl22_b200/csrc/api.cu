@@ -449,6 +449,8 @@ int ganns_build(const float* points, int64_t n, int d, int metric, int degree,
   if (d_min >= n) return fail(GANNS_EINVAL, "d_min must be < n");
   if (l_build < d_min || l_build > 1024) return fail(GANNS_EINVAL, "l_build must be in [d_min, 1024]");
   if (e_build < 1 || e_build > l_build) return fail(GANNS_EINVAL, "e_build must be in [1, l_build]");
+  const int l_local = p && p->l_local > 0 ? p->l_local : l_build;
+  if (l_local < d_min || l_local > l_build) return fail(GANNS_EINVAL, "l_local must be in [d_min, l_build]");
   int64_t S = p && p->group_size > 0 ? p->group_size : 0;
   if (S == 0) S = auto_group_size(n);
   if (S > n) S = n;
@@ -464,6 +466,8 @@ int ganns_build(const float* points, int64_t n, int d, int metric, int degree,
   a.d_min = d_min;
   a.l_build = l_build;
   a.e_build = e_build;
+  a.l_local = l_local;
+  a.e_local = std::min(e_build, l_local);
   a.group_size = S;
   a.max_rounds = p ? (p->stop_after_phase1 ? 0 : (p->max_rounds > 0 ? p->max_rounds : -1)) : -1;
   a.out_nbr = (*out)->nbr;
@@ -581,6 +585,8 @@ int ganns_build_hnsw(const float* points, int64_t n, int d, int metric, int degr
     a.d_min = d_min;
     a.l_build = l_build;
     a.e_build = e_build;
+    a.l_local = l_build;   // HNSW layers: Phase 1 at l_build (the oracle's HNSW has no l_local)
+    a.e_local = e_build;
     int64_t S = p && p->group_size > 0 ? p->group_size : 0;
     if (S == 0) S = auto_group_size(layer_n[j]);
     a.group_size = std::max<int64_t>(1, std::min<int64_t>(S, layer_n[j]));

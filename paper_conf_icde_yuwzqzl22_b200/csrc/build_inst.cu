@@ -101,6 +101,7 @@ struct BuildDev {
   int32_t* gpid;
   float* gpd;
   int d_min, l_build, e_build;
+  int l_local, e_local;   // Phase-1 searches on the local graphs (<= l_build)
   unsigned long long* stats;   // [3] iterations, comps, searches
 };
 
@@ -136,7 +137,7 @@ phase1_kernel(BuildDev B, int64_t group_size, int64_t ngroups,
     // Step 1 (line 5): v.N, v.N' := Search(G_i, v, d_min), entry = group's first vertex
     SearchStats st;
     const int cnt = warp_search<NV4, TPL, L2, true>(B.g, B.g.X + size_t(v) * d, int32_t(lo),
-                                                    B.l_build, B.e_build, ws, st);
+                                                    B.l_local, B.e_local, ws, st);
     add_stats(B.stats, st, lane);
     const int m = cnt < B.d_min ? cnt : B.d_min;
     for (int j = lane; j < m; j += 32) {
@@ -395,6 +396,8 @@ static int build_t(BuildArgs& a, cudaStream_t s) {
   B.d_min = dm;
   B.l_build = a.l_build;
   B.e_build = a.e_build;
+  B.l_local = a.l_local > 0 ? a.l_local : a.l_build;
+  B.e_local = a.e_local > 0 ? a.e_local : a.e_build;
   B.stats = stats.p;
   const size_t smem =
       size_t(kBuildWarps) * warp_smem_bytes(a.l_build, TPL, NV4, a.d / 4, kBuildStageRounds);

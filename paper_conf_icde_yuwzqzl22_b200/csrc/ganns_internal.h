@@ -102,6 +102,7 @@ struct BuildArgs {
   const float* X;
   int64_t n;
   int d, metric, d_max, d_min, l_build, e_build;
+  int l_local = 0, e_local = 0;   // Phase-1 searches (0: l_build / e_build)
   int64_t group_size;
   int max_rounds;       // < 0: all
   int32_t* out_nbr;     // device [n][d_max]

@@ -91,3 +91,13 @@ def test_build_c1_parity_and_quality():
     assert (ids.cpu().numpy() == oi).all() and (dists.cpu().numpy() == od).all()
     gt, _ = oracle.bruteforce(X, Q, 10)
     assert oracle.recall(oi, gt) > 0.8
+
+
+@pytest.mark.parametrize("l_local", [16, 40])
+def test_build_parity_l_local(l_local):
+    """Phase-1 searches at l_local < l_build (R-C13): bit-exact vs the oracle."""
+    cfg = syn.with_size(syn.CONFIGS["C1"], n=4000)
+    X = syn.points(cfg)
+    ref, _, _ = oracle.alg2(X, 8, 16, 256, l_build=64, l_local=l_local)
+    _, adj = gpu_build(X, 16, l_build=64, group_size=256, l_local=l_local)
+    assert (adj == ref).all()

@@ -276,6 +276,28 @@ def test_alg2_max_rounds_zero_is_union_of_local_graphs():
         assert (ids[g * 300:(g + 1) * 300] == sub).all()
 
 
+def test_alg2_l_local_is_phase1_only():
+    """l_local (R-C13) sets the list length of the Phase-1 searches only: (1) with
+    max_rounds = 0 the result is each group's sequential NSW at list length l_local;
+    (2) once l_local >= the group size every local search is exhaustive (l >= |G_i|,
+    connected local graph: pin P3), so any such l_local gives the same graph; (3) a
+    short l_local still changes the local graphs (the parameter is live)."""
+    X = syn.points(syn.with_size(syn.CONFIGS["C1"], n=900))
+    ids, _, _ = oracle.alg2(X, 8, 16, 300, l_build=64, max_rounds=0, l_local=16)
+    for g in range(3):
+        sub, _, _ = oracle.nsw_seq(X[g * 300:(g + 1) * 300], 8, 16, l_build=16)
+        sub = np.where(sub >= 0, sub + g * 300, -1)
+        assert (ids[g * 300:(g + 1) * 300] == sub).all()
+    a, _, _ = oracle.alg2(X, 8, 16, 60, l_build=96, l_local=64)
+    b, _, _ = oracle.alg2(X, 8, 16, 60, l_build=96, l_local=96)
+    assert (a == b).all()
+    c, _, _ = oracle.alg2(X, 8, 16, 300, l_build=64, l_local=8)
+    d, _, _ = oracle.alg2(X, 8, 16, 300, l_build=64)
+    assert (c != d).any()
+    with pytest.raises(Exception):
+        oracle.alg2(X, 8, 16, 300, l_build=64, l_local=128)   # l_local > l_build
+
+
 # ------------------------------------- P8: Fig. 12 quality (statistical)
 def test_alg2_quality_matches_sequential_nsw():
     """Fig. 12: GGraphCon's graph is as good as the sequential NSW
