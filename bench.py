@@ -202,7 +202,7 @@ class BenchIndex:
         self.g, self.cfg, self.Xd = g, cfg, Xd
         self.hnsw = cfg.name == "C4"
         if self.hnsw:
-            levels = syn.hnsw_levels(cfg.n, cfg.degree // 2, 1)
+            levels = syn.hnsw_levels(Xd.shape[0], cfg.degree // 2, 1)
             self.idx = g.build_hnsw(Xd, levels, metric=cfg.metric, degree=cfg.degree,
                                     l_build=l_build)
             self.graph = self.idx.base
@@ -389,16 +389,28 @@ def run_ours(args):
     Qds = [Qd_all[b * nq:(b + 1) * nq] for b in range(B)]
     torch.cuda.synchronize()
 
-    # ---- GGraphCon build (timed wall clock on device-resident points)
-    t0 = time.perf_counter()
-    index = BenchIndex(g, cfg, Xd, args.l_build, args.l_local)
+    # exact ground truth first: it also brings the GPU out of its idle clocks before
+    # the timed build
+    gt = ground_truth(torch, Xd, Qd_all, k, cfg.metric)
+    # untimed warm-up build on a 20K-point prefix (loads the build kernels' modules)
+    BenchIndex(g, cfg, Xd[:20000].contiguous(), args.l_build, args.l_local)
     torch.cuda.synchronize()
-    build_s = time.perf_counter() - t0
+
+    # ---- GGraphCon build (wall clock on device-resident points; median of 3 builds,
+    # the builds are deterministic, the last one is searched)
+    build_all = []
+    for _ in range(3):
+        index = None
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        index = BenchIndex(g, cfg, Xd, args.l_build, args.l_local)
+        torch.cuda.synchronize()
+        build_all.append(time.perf_counter() - t0)
+    build_s = statistics.median(build_all)
     b_iters, b_comps, b_searches, b_rounds = index.build_stats
 
     # ---- (l, e) operating point over every query the timed steps search (see
     # select_operating_point); candidates timed as the steps are (pipelined)
-    gt = ground_truth(torch, Xd, Qd_all, k, cfg.metric)
     pipe = Pipeline(torch, index, Qds, k, args.streams)
     l_star, e_star, sweep, chosen = select_operating_point(
         torch, index, Qd_all, gt, k, args.target,
@@ -496,6 +508,7 @@ def run_ours(args):
                           f"{nq}-query batches"),
                    "parallelism": f"replicated graph, query data-parallel x{world}"},
         "build_seconds": round(build_s, 4),
+        "build_seconds_all": [round(x, 4) for x in build_all],
         "build_params": {"degree": cfg.degree, "d_min": cfg.degree // 2, "l_build": args.l_build,
                          "l_local": (None if index.hnsw else min(args.l_local, args.l_build) or
                                      args.l_build),
@@ -563,6 +576,10 @@ def run_sharded(args):
     Qd = torch.from_numpy(Q).to(dev)
     nsub = min(1000, len(Q))                 # recall measured on a fixed query subset
     shards, build_s, gt_parts = [], 0.0, []
+    # untimed warm-up build (module load, GPU out of idle clocks)
+    g.build(torch.from_numpy(syn.points(cfg, 0, 20000)).to(dev), metric=cfg.metric,
+            degree=cfg.degree, l_build=args.l_build, l_local=min(args.l_local, args.l_build))
+    torch.cuda.synchronize()
     for s in mine:
         Xs = torch.from_numpy(syn.points(cfg, s * per, (s + 1) * per)).to(dev)
         torch.cuda.synchronize()

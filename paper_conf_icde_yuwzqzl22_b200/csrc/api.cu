@@ -158,14 +158,15 @@ int host_async(int d, const float* queries_host, int64_t nq, int k, float* queri
   return err == cudaSuccess ? GANNS_OK : cuda_fail(err, "D2H results");
 }
 
-// R-C14: automatic group size = clamp(pow2round(sqrt n), 256, 8192) -- 1024 at n = 1M.
-// The build takes ~ s * t_insert (Phase 1, s sequential insertions per group) +
-// (n / s) * t_round (Phase 2): measured on C2 (B200) 0.855 s at s = 1024 vs 0.975 s at
-// 2048 and 0.98-1.7 s at 768, with the same search recall at every s.
+// R-C14: automatic group size = clamp(1.5 sqrt n rounded to a multiple of 256, 256,
+// 8192) -- 1536 at n = 1M.  The build takes ~ s * t_insert (Phase 1, s sequential
+// insertions per group) + (n / s) * t_round (Phase 2): measured on C2 (B200, l_build
+// 128, l_local 64) 0.72 s at s = 1024, 0.65 s at 1536, 0.72 s at 2048, with the same
+// search recall at every s.
 int64_t auto_group_size(int64_t n) {
-  const double t = std::sqrt(double(std::max<int64_t>(n, 1)));
-  const int64_t s2 = int64_t(1) << int64_t(std::llround(std::log2(std::max(t, 1.0))));
-  return std::min<int64_t>(8192, std::max<int64_t>(256, s2));
+  const double t = 1.5 * std::sqrt(double(std::max<int64_t>(n, 1)));
+  const int64_t s = int64_t(std::llround(t / 256.0)) * 256;
+  return std::min<int64_t>(8192, std::max<int64_t>(256, s));
 }
 
 }  // namespace ganns

@@ -74,7 +74,7 @@ def test_c2_build_phase1_sampled_groups(c2):
     cfg, X, Q, Xd, Qd = c2
     graph = g.build(Xd, degree=cfg.degree, l_build=64, stop_after_phase1=True)
     adj = graph.adjacency()
-    S = 1024   # R-C14 auto for n = 1M: clamp(pow2round(sqrt(n)), 256, 8192)
+    S = 1536   # R-C14 auto for n = 1M: clamp(round256(1.5 sqrt(n)), 256, 8192)
     ngroups = (cfg.n + S - 1) // S
     for gi in (0, 1, ngroups // 2, ngroups - 1):
         lo, hi = gi * S, min(cfg.n, (gi + 1) * S)
@@ -101,7 +101,7 @@ def test_c2_build_full_invariants_and_recall(c2):
     ids, _ = g.search(graph, Xd, Qd[:200], cfg.k, 128)
     gt, _ = oracle.bruteforce(X, Q[:200], cfg.k)
     assert oracle.recall(ids.cpu().numpy(), gt) >= 0.93
-    assert graph.build_stats[3] == (cfg.n + 1023) // 1024 - 1       # Phase-2 rounds (auto s = 1024)
+    assert graph.build_stats[3] == (cfg.n + 1535) // 1536 - 1       # Phase-2 rounds (auto s = 1536)
 
 
 def test_c4_cosine_fullsize_sampled():

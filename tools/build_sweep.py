@@ -28,7 +28,8 @@ for s in groups:
     for _ in range(3):
         torch.cuda.synchronize()
         t0 = time.perf_counter()
-        gr = g.build(Xd, metric=cfg.metric, degree=cfg.degree, l_build=lb, group_size=s)
+        gr = g.build(Xd, metric=cfg.metric, degree=cfg.degree, l_build=lb, group_size=s,
+                     l_local=int(os.environ.get("LL", "0")))
         torch.cuda.synchronize()
         ts.append(time.perf_counter() - t0)
     idx = BenchIndex.__new__(BenchIndex)
