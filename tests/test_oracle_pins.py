@@ -316,6 +316,46 @@ def test_alg2_quality_matches_sequential_nsw():
     assert rec["naive"] < rec["alg2"] - 0.02, rec
 
 
+@pytest.mark.parametrize("batch", [1, 2, 5])
+def test_naive_parallel_exact_regime_definition(batch):
+    """GNaiveParallel (P:240-242) with l_build >= n and d_max >= n - 1, checked
+    against its definition written out with BFS + numpy lexsort: every point of a
+    batch takes the d_min nearest of the points reachable from entry 0 in the
+    graph as it stood before the batch (an l >= n search returns exactly the
+    reachable set, P3), and the batch's links are added afterwards, both ways."""
+    for seed in range(8):
+        n, d_min = 23, 3
+        X = syn.random_int_points(n, 3, 0, 4, 700 + seed)
+        ids, dists = oracle.naive_parallel(X, d_min, n - 1, batch, l_build=n + 1)
+        D = ((X[:, None, :].astype(np.int64) - X[None].astype(np.int64)) ** 2).sum(-1)
+        adj = [set() for _ in range(n)]
+        for b0 in range(0, n, batch):
+            b1 = min(b0 + batch, n)
+            reach = set()
+            if b0 > 0:
+                reach, todo = {0}, [0]
+                while todo:
+                    u = todo.pop()
+                    for w in adj[u]:
+                        if w not in reach:
+                            reach.add(w)
+                            todo.append(w)
+            cand = np.array(sorted(reach), np.int64)
+            new = []
+            for v in range(b0, b1):
+                if len(cand):
+                    f = cand[np.lexsort((cand, D[v, cand]))[:d_min]]
+                    new += [(v, int(u)) for u in f]
+            for v, u in new:
+                adj[v].add(u)
+                adj[u].add(v)
+        for v in range(n):
+            row = ids[v][ids[v] >= 0].tolist()
+            assert sorted(row, key=lambda u: (D[v, u], u)) == row, (seed, v)
+            assert set(row) == adj[v], (seed, v)
+            assert dists[v][:len(row)].tolist() == [float(D[v, u]) for u in row]
+
+
 # ------------------------------- shard merge (SURVEY §8(e)) == global brute force
 @pytest.mark.parametrize("W", [1, 2, 3, 8])
 def test_merge_topk_of_exact_shards_is_global_bruteforce(W):
