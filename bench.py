@@ -479,8 +479,10 @@ def run_ours(args):
     if os.path.exists(tp):
         with open(tp) as f:
             tr = json.load(f)
-        if tr.get("config") == args.config and tr.get("l") == l_star and tr.get("e", l_star) == e_star:
-            traffic = tr.get("dram_bytes_per_launch")
+        for ent in tr.get("entries", [tr]):
+            if (ent.get("config") == args.config and ent.get("l") == l_star
+                    and ent.get("e", l_star) == e_star):
+                traffic = ent.get("dram_bytes_per_launch")
 
     line = {
         "metric": "queries/sec at recall@10=0.95",

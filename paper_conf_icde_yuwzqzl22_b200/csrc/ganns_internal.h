@@ -32,6 +32,14 @@ constexpr int kSearchPool = GANNS_SEARCH_POOL;     // shared stage buffers per C
 #endif
 constexpr int kMinBlocksPerSM = GANNS_MIN_BLOCKS; // register budget: <= 85 regs/thread (24 warps per SM);
                                     // the TMA stage (8 KB/warp at d=128) allows ~22 warps
+#ifndef GANNS_MIN_BLOCKS_WIDE
+#define GANNS_MIN_BLOCKS_WIDE (16 / GANNS_SEARCH_WARPS)
+#endif
+// d > 128 (NV4 >= 2): the TMA stage (>= 16.5 KB/warp) caps residency at <= 14 warps
+// per SM, so the register budget may grow to 128/thread (16 warps) at no occupancy
+// cost; at 80 the C4 (d = 200, HNSW) instance spilled 268 B/thread to local memory
+// (ncu: 62 M local store requests per launch, 566 MB of DRAM writes).
+constexpr int kMinBlocksWide = GANNS_MIN_BLOCKS_WIDE;
 
 void set_error(const std::string& msg);
 int fail(int status, const std::string& msg);

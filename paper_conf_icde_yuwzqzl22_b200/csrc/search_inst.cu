@@ -34,7 +34,7 @@ struct HnswUpper {
   const int32_t* perm;
 };
 template <int NV4, int TPL, bool L2, bool HNSW>
-__global__ void __launch_bounds__(kSearchWarps * 32, kMinBlocksPerSM)
+__global__ void __launch_bounds__(kSearchWarps * 32, NV4 == 1 ? kMinBlocksPerSM : kMinBlocksWide)
 search_kernel(GraphView g, const float* __restrict__ Q, int64_t nq, int k, int l, int e,
               int32_t entry, int32_t* __restrict__ out_ids, float* __restrict__ out_dists,
               uint32_t* __restrict__ stats, int32_t* __restrict__ ticket,
