@@ -53,6 +53,8 @@ def lib():
         _lib.ora_alg2.argtypes = [P, i64, i32, i32, i32, i32, i32, i32, i64, i32, i32, P, P, P]
         _lib.ora_alg2_ex.argtypes = [P, i64, i32, i32, i32, i32, i32, i32, i32, i64, i32, i32, P,
                                      P, P]
+        _lib.ora_alg2_mt.argtypes = [P, i64, i32, i32, i32, i32, i32, i32, i32, i64, i32, i32, P,
+                                     P, P, i32]
         _lib.ora_naive_parallel.argtypes = [P, i64, i32, i32, i32, i32, i32, i32, i64, P, P]
         _lib.ora_merge_topk.argtypes = [P, P, i32, i64, i32, P, P]
         _lib.ora_knn_descent.argtypes = [P, i64, i32, i32, i32, P, i32, P, P, P]
@@ -62,7 +64,8 @@ def lib():
         _lib.ora_hnsw_search.argtypes = [P, P, i32, P, P, i64, i32, P, i32, i32, P, i64, i32,
                                          i32, i32, P, P, P, P]
         for f in ("ora_hnsw_build", "ora_hnsw_search", "ora_merge_topk", "ora_search_one", "ora_search_batch", "ora_alg1", "ora_bruteforce",
-                  "ora_nsw_seq", "ora_alg2", "ora_alg2_ex", "ora_naive_parallel"):
+                  "ora_nsw_seq", "ora_alg2", "ora_alg2_ex", "ora_alg2_mt",
+                  "ora_naive_parallel"):
             getattr(_lib, f).restype = ct.c_int
     return _lib
 
@@ -178,17 +181,19 @@ def nsw_seq(X, d_min, d_max, l_build=64, e_build=0, exact=False, metric="l2"):
 
 
 def alg2(X, d_min, d_max, group_size, l_build=64, e_build=0, exact=False, metric="l2",
-         max_rounds=-1, l_local=0):
+         max_rounds=-1, l_local=0, threads=1):
     """O5 Algorithm 2.  Returns (ids [n,d_max], dists [n,d_max], stats[3]).  l_local
-    (0 = l_build): list length of the Phase-1 searches on the local graphs (R-C13)."""
+    (0 = l_build): list length of the Phase-1 searches on the local graphs (R-C13).
+    threads > 1 splits the units the paper runs in parallel (Phase-1 groups, the
+    searches of a Phase-2 round) over POSIX threads; the result does not depend on it."""
     X = _f32(X)
     n = X.shape[0]
     ids = np.empty((n, d_max), np.int32)
     dists = np.empty((n, d_max), np.float32)
     st = np.zeros(3, np.uint32)
-    _check(lib().ora_alg2_ex(_p(X), n, X.shape[1], METRICS[metric], d_min, d_max, l_build,
+    _check(lib().ora_alg2_mt(_p(X), n, X.shape[1], METRICS[metric], d_min, d_max, l_build,
                              e_build, l_local, group_size, int(exact), max_rounds, _p(ids),
-                             _p(dists), _p(st)))
+                             _p(dists), _p(st), max(1, int(threads))))
     return ids, dists, st
 
 
