@@ -174,7 +174,7 @@ def nsw_seq(X, d_min, d_max, l_build=64, e_build=0, exact=False, metric="l2"):
     n = X.shape[0]
     ids = np.empty((n, d_max), np.int32)
     dists = np.empty((n, d_max), np.float32)
-    st = np.zeros(3, np.uint32)
+    st = np.zeros(3, np.uint64)
     _check(lib().ora_nsw_seq(_p(X), n, X.shape[1], METRICS[metric], d_min, d_max, l_build,
                              e_build, int(exact), _p(ids), _p(dists), _p(st)))
     return ids, dists, st
@@ -190,7 +190,7 @@ def alg2(X, d_min, d_max, group_size, l_build=64, e_build=0, exact=False, metric
     n = X.shape[0]
     ids = np.empty((n, d_max), np.int32)
     dists = np.empty((n, d_max), np.float32)
-    st = np.zeros(3, np.uint32)
+    st = np.zeros(3, np.uint64)
     _check(lib().ora_alg2_mt(_p(X), n, X.shape[1], METRICS[metric], d_min, d_max, l_build,
                              e_build, l_local, group_size, int(exact), max_rounds, _p(ids),
                              _p(dists), _p(st), max(1, int(threads))))

@@ -10,11 +10,11 @@ that independent work units parallelise directly.
   is needed for throughput; :func:`search_replicated` all-gathers the slices
   when the caller wants the whole result on every rank.
 
-* Sharded base set (BASELINE configs[4], DEEP100M-shaped): rank r holds rows
-  [r*n/W, (r+1)*n/W) and its own graph over them; every rank searches ALL
-  queries on its shard, turns local ids into global ids, and one all-gather of
-  the [nq, k] (id, dist) lists is followed by the K6 merge (ganns_merge_topk):
-  the k smallest (dist, global id) over all shards.
+* Sharded base set (BASELINE configs[4], DEEP100M-shaped): the rows are split
+  into shards, each with its own graph; a rank holds one or more shards, searches
+  ALL queries on each, turns local ids into global ids, and one
+  all_gather_into_tensor of the stacked [S, nq, k] (id, dist) lists is followed by
+  the K6 merge (ganns_merge_topk): the k smallest (dist, global id) over all shards.
 
 The per-shard search / merge functions are injected, so the same orchestration
 runs the sm_100a kernels on GPUs and is exercised on CPU by the gloo tests.
@@ -72,46 +72,82 @@ def search_replicated(search_fn: SearchFn, queries: torch.Tensor, gather: bool =
 
 
 class ShardedIndex:
-    """One shard of a base set split across ranks; `search` returns the global top-k.
+    """The shards of a base set held by this rank; `search` returns the global top-k.
 
-    search_fn(queries) -> (local ids, dists) of this rank's shard (ids in
-    [0, shard size), -1 = empty); offset_fn(ids, offset) makes them global in
-    place; merge_fn(ids[W,nq,k], dists[W,nq,k]) -> global (ids, dists) [nq, k].
+    shards: [(global_offset, search_fn)] -- this rank's shards (every rank holds
+    the same number of shards; shard s lives on rank s % W in the bench, any
+    placement works).  search_fn(queries) -> (local ids, dists) [nq, k] of that
+    shard (ids in [0, shard size), -1 = empty); offset_fn(ids, offset) makes them
+    global in place; merge_fn(ids [S, nq, k], dists [S, nq, k]) -> global
+    (ids, dists) [nq, k].  streams (optional, one per concurrent shard search):
+    shard j's search + offset run on streams[j % len(streams)] so consecutive
+    shard searches overlap on the device; the exchange waits for all of them.
+
+    The one exchange step is an all_gather_into_tensor of the stacked per-shard
+    lists ([S_local, nq, k] ids and dists per rank) -- 800 KB per shard at 10K
+    queries, k = 10 -- followed by the K6 merge on every rank.
     """
 
-    def __init__(self, n_total: int, search_fn: SearchFn, merge_fn: MergeFn,
-                 offset_fn: Callable[[torch.Tensor, int], torch.Tensor], group=None):
+    def __init__(self, shards, merge_fn: MergeFn,
+                 offset_fn: Callable[[torch.Tensor, int], torch.Tensor], group=None,
+                 streams=None):
         self.rank, self.world = _world(group)
         self.group = group
-        self.lo, self.hi = shard_bounds(n_total, self.rank, self.world)
-        self.search_fn = search_fn
+        self.shards = list(shards)
+        if not self.shards:
+            raise ValueError("a rank must hold at least one shard")
         self.merge_fn = merge_fn
         self.offset_fn = offset_fn
+        self.streams = list(streams) if streams else None
+
+    def local(self, queries: torch.Tensor):
+        """Every local shard searched, ids made global: stacked [S_local, nq, k]."""
+        if self.streams is None:
+            outs = []
+            for off, fn in self.shards:
+                ids, dists = fn(queries)
+                outs.append((self.offset_fn(ids, off), dists))
+        else:
+            cur = torch.cuda.current_stream()
+            ev0 = torch.cuda.Event()
+            ev0.record(cur)
+            outs = [None] * len(self.shards)
+            for j, (off, fn) in enumerate(self.shards):
+                st = self.streams[j % len(self.streams)]
+                st.wait_event(ev0)
+                with torch.cuda.stream(st):
+                    ids, dists = fn(queries)
+                    outs[j] = (self.offset_fn(ids, off), dists)
+            for st in self.streams:
+                ev = torch.cuda.Event()
+                ev.record(st)
+                cur.wait_event(ev)
+        return torch.stack([o[0] for o in outs]), torch.stack([o[1] for o in outs])
 
     def search(self, queries: torch.Tensor):
-        ids, dists = self.search_fn(queries)
-        ids = self.offset_fn(ids, self.lo)
-        if self.world == 1:
-            return self.merge_fn(ids[None], dists[None])
-        # the one exchange step: all-gather of every shard's [nq, k] lists
-        gi = [torch.empty_like(ids) for _ in range(self.world)]
-        gd = [torch.empty_like(dists) for _ in range(self.world)]
-        dist.all_gather(gi, ids.contiguous(), group=self.group)
-        dist.all_gather(gd, dists.contiguous(), group=self.group)
-        return self.merge_fn(torch.stack(gi), torch.stack(gd))
+        ids, dists = self.local(queries)
+        if self.world > 1:
+            gi = ids.new_empty((self.world * ids.shape[0],) + tuple(ids.shape[1:]))
+            gd = dists.new_empty((self.world * dists.shape[0],) + tuple(dists.shape[1:]))
+            dist.all_gather_into_tensor(gi, ids.contiguous(), group=self.group)
+            dist.all_gather_into_tensor(gd, dists.contiguous(), group=self.group)
+            ids, dists = gi, gd
+        return self.merge_fn(ids, dists)
 
 
-def gpu_sharded_index(graph, points_shard: torch.Tensor, n_total: int, k: int, l: int,
-                      e: int = 0, group=None) -> ShardedIndex:
-    """ShardedIndex wired to the sm_100a kernels: K1 search on the local shard graph,
-    in-place id offset, K6 merge (all through libganns.so)."""
+def gpu_sharded_index(shards, k: int, l: int, e: int = 0, group=None,
+                      streams=None) -> ShardedIndex:
+    """ShardedIndex wired to the sm_100a kernels: shards = [(global_offset, graph,
+    points_shard)]; K1 search on each local shard graph, in-place id offset, K6
+    merge (all through libganns.so)."""
     from . import search, offset_ids, merge_topk
 
-    def _search(q):
-        return search(graph, points_shard, q, k, l, e=e)
+    def _fn(graph, pts):
+        return lambda q: search(graph, pts, q, k, l, e=e)
 
-    return ShardedIndex(n_total, _search, lambda i, d: merge_topk(i, d),
-                        lambda ids, off: offset_ids(ids, off), group=group)
+    return ShardedIndex([(off, _fn(gr, pts)) for off, gr, pts in shards],
+                        lambda i, d: merge_topk(i, d), lambda ids, off: offset_ids(ids, off),
+                        group=group, streams=streams)
 
 
 def gpu_replicated_search(graph, points: torch.Tensor, queries: torch.Tensor, k: int, l: int,

@@ -60,11 +60,24 @@ def _worker(rank, world, port, out_dir):
     def offset(i, off):
         return torch.where(i >= 0, i + off, i)
 
-    idx = gd.ShardedIndex(len(X), search_shard, merge, offset)
+    idx = gd.ShardedIndex([(lo, search_shard)], merge, offset)
     si, sd = idx.search(torch.from_numpy(Q))
+    # two shards per rank (the bench's C5 layout on fewer GPUs than shards):
+    # shard s = 2 * rank + j covers rows quarter s
+    quart = [gd.shard_bounds(len(X), s, 2 * world) for s in range(2 * world)]
+    mine = []
+    for s in (2 * rank, 2 * rank + 1):
+        a, b = quart[s]
+        nb, _, _ = oracle.alg2(X[a:b], 8, 16, 128, l_build=32)
+
+        def fn(q, nb=nb, a=a, b=b):
+            i, d = oracle.search(nb, X[a:b], q.numpy(), k, l)
+            return torch.from_numpy(i), torch.from_numpy(d)
+        mine.append((a, fn))
+    mi2, md2 = gd.ShardedIndex(mine, merge, offset).search(torch.from_numpy(Q))
     t = gd.max_over_ranks(float(rank + 1))
     np.savez(os.path.join(out_dir, f"r{rank}.npz"), ri=ri.numpy(), rd=rd.numpy(),
-             si=si.numpy(), sd=sd.numpy(), t=t)
+             si=si.numpy(), sd=sd.numpy(), mi2=mi2.numpy(), md2=md2.numpy(), t=t)
     dist.destroy_process_group()
 
 
@@ -105,6 +118,17 @@ def test_sharded_equals_sequential_shards_and_merge(results):
     for r in results:
         assert (r["si"] == mi).all() and (r["sd"] == md).all()
         assert float(r["t"]) == 2.0        # max over ranks
+    # 4 shards over 2 ranks == 4 sequential shard searches + the oracle's merge
+    parts_i, parts_d = [], []
+    for s in range(4):
+        a, b = gd.shard_bounds(len(X), s, 4)
+        nb, _, _ = oracle.alg2(X[a:b], 8, 16, 128, l_build=32)
+        i, d = oracle.search(nb, X[a:b], Q, 10, 48)
+        parts_i.append(np.where(i >= 0, i + a, -1))
+        parts_d.append(d)
+    mi4, md4 = oracle.merge_topk(np.stack(parts_i), np.stack(parts_d))
+    for r in results:
+        assert (r["mi2"] == mi4).all() and (r["md2"] == md4).all()
     # sharding can only help recall at equal l (each shard keeps its own top-l)
     gt, _ = oracle.bruteforce(X, Q, 10)
     nbr, _, _ = oracle.alg2(X, 8, 16, 256, l_build=32)
