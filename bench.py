@@ -63,6 +63,12 @@ def parse():
                     help="CUDA streams the steps alternate over (1 = serialised launches)")
     ap.add_argument("--shard-rows", type=int, default=0,
                     help="C5 only: rows per shard (default: n / shards = 12.5M)")
+    ap.add_argument("--scaling", default="weak", choices=["weak", "strong"],
+                    help="weak: every rank searches its own batches; strong: each step's "
+                         "batch is split over the ranks (dist.query_slice)")
+    ap.add_argument("--proxy-worlds", default="2,4,8",
+                    help="N=1 only: strong-scaling proxy -- time each of the W slices of the "
+                         "fixed batch alone on this GPU (max over slices), per W")
     return ap.parse_args()
 
 
@@ -231,13 +237,24 @@ class BenchIndex:
         return out
 
     def oracle_search(self, X, Q, k, l, e, threads):
+        """The oracle on the same graph: (ids, dists, stats [iters, comps, drops,
+        merged]).  The HNSW oracle search is single-threaded."""
         import oracle
         if not self.hnsw:
-            return oracle.search(self.graph.adjacency(), X, Q, k, l, e=e, metric=self.cfg.metric,
-                                 threads=threads)
+            if not hasattr(self, "_adj"):
+                self._adj = self.graph.adjacency()
+            return oracle.search(self._adj, X, Q, k, l, e=e, metric=self.cfg.metric,
+                                 threads=threads, stats=True)
         h = self._oracle_index()
-        ids, dists, _ = oracle.hnsw_search(h, X, Q, k, l, e=e, metric=self.cfg.metric)
-        return ids, dists
+        ids, dists, _, st = oracle.hnsw_search(h, X, Q, k, l, e=e, metric=self.cfg.metric,
+                                               stats=True)
+        return ids, dists, st
+
+    def descent_stats(self, Qd, k, l, e):
+        """HNSW: per query (iterations, distance computations) of the greedy descent
+        through the upper layers (R-H1), counted by the fused kernel itself."""
+        return self.g.hnsw_search(self.idx, self.Xd, Qd, k, l, e=e, stats=True,
+                                  descent_stats=True)[3]
 
     def _oracle_index(self):
         if not hasattr(self, "_oi"):
@@ -256,9 +273,11 @@ class Pipeline:
     the start of the next one.  Device-timed with CUDA events bracketing all
     streams."""
 
-    def __init__(self, torch, index, Qds, k, nstreams):
-        self.torch, self.index, self.Qds, self.k = torch, index, Qds, k
-        nq = Qds[0].shape[0]
+    def __init__(self, torch, index, Qds, k, nstreams, lo=0, hi=None):
+        self.torch, self.index, self.k = torch, index, k
+        hi = Qds[0].shape[0] if hi is None else hi
+        self.Qds = [q[lo:hi] for q in Qds]          # this rank's slice of every batch
+        nq = hi - lo
         dev = Qds[0].device
         self.streams = [torch.cuda.Stream(device=dev) for _ in range(max(1, nstreams))]
         self.outs = [(torch.empty((nq, k), dtype=torch.int32, device=dev),
@@ -363,10 +382,156 @@ def select_operating_point(torch, index, Qd, gt, k, target, timer):
     return l_star, e_star, sweep, chosen
 
 
+def dram_counters_usable():
+    """The CUPTI profiler cannot be shared with ncu / nsys, which inject themselves
+    through CUDA_INJECTION64_PATH (e.g. the launch-list pass under ncu)."""
+    return not os.environ.get("CUDA_INJECTION64_PATH")
+
+
+def measure_dram(run, device):
+    """DRAM traffic of run() (which enqueues work and synchronises) from the
+    hardware counters: CUPTI range profiler, one pass, user range (tools/dramprof),
+    so the kernels run exactly as in the timed pass -- concurrent streams included."""
+    if not dram_counters_usable():
+        return {"error": "another profiler is attached (CUDA_INJECTION64_PATH)"}
+    from tools.dramprof import DramRegion
+    with DramRegion(device) as r:
+        secs = run()
+    if r.read_bytes is None:
+        return {"error": r.error}
+    return {"read": r.read_bytes, "write": r.write_bytes,
+            "l2_read": r.l2_read_sectors * 32.0, "seconds": secs}
+
+
+def read_peak_gbps(torch, dev, gib=2):
+    """Read-only DRAM bandwidth of a torch reduction over `gib` GiB (context for the
+    copy peak of MEASURED_PEAKS.json, which mixes reads and writes; the search
+    traffic is > 99.9 % reads)."""
+    x = torch.ones((gib << 28,), dtype=torch.float32, device=dev)
+    best = None
+    for _ in range(6):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        x.sum()
+        e1.record()
+        e1.synchronize()
+        t = e0.elapsed_time(e1) / 1e3
+        best = t if best is None else min(best, t)
+    gbps = x.numel() * 4 / best / 1e9
+    del x
+    torch.cuda.empty_cache()
+    return round(gbps, 1)
+
+
+def roofline(alg_bytes, launch_s, dram, launches, peak, peak_kind, kernel, duration):
+    """The line's roofline object.  `achieved` / `frac` / `traffic` are DRAM bytes
+    measured by the hardware counters over `launches` launches of the timed
+    configuration, per launch, over the launch duration of the timed pass.  The
+    SURVEY §8(d) algorithmic bytes (every gathered row, lazy-check re-reads
+    included) are reported beside them: rows served by the 126 MB L2 count
+    there too, so alg_frac is an L2-level figure and can exceed 1."""
+    alg = alg_bytes / launch_s / 1e9
+    r = {"bound": "hbm", "peak": peak, "unit": "GB/s", "peak_kind": peak_kind, "kernel": kernel,
+         "duration": duration, "alg_bytes_per_launch": int(alg_bytes), "alg_GBps": round(alg, 1),
+         "alg_frac": round(alg / peak, 4),
+         "alg_note": "SURVEY 8(d) algorithmic bytes incl. lazy-check re-reads (P:191); "
+                     "L2-served rows count, so this is an L2-level figure"}
+    if "error" not in dram:
+        per = (dram["read"] + dram["write"]) / launches
+        ach = per / launch_s / 1e9
+        r.update(achieved=round(ach, 1), frac=round(ach / peak, 4), traffic=int(per),
+                 traffic_read=int(dram["read"] / launches),
+                 traffic_write=int(dram["write"] / launches),
+                 l2_read_bytes_per_launch=int(dram["l2_read"] / launches),
+                 dram_over_alg=round(per / alg_bytes, 4),
+                 achieved_kind="measured DRAM bytes per launch / launch duration",
+                 traffic_source=(f"hardware counters dram__bytes_read.sum + dram__bytes_write.sum "
+                                 f"(CUPTI range profiler, one pass) over {launches} launches of "
+                                 f"the timed configuration in this run"),
+                 profiled_pass_s=round(dram["seconds"], 6))
+    else:
+        r.update(achieved=round(alg, 1), frac=round(alg / peak, 4), traffic=None,
+                 achieved_kind=f"algorithmic (DRAM counters unavailable: {dram['error']})")
+    return r
+
+
+def cpu_model():
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return None
+
+
+def parity_report(gpu, ora, exact, gt=None):
+    """Element-by-element comparison of the GPU's results with the oracle's on the
+    same queries, graph and (l, e).  gpu = (ids, dists, stats[iters, comps,
+    merged]); ora = (ids, dists, stats[iters, comps, drops, merged]).  exact
+    (integer grid): ids, dists and counters bit-identical.  Otherwise (cosine):
+    |d_gpu - d_ora| <= 1e-5 |d| + 1e-6, id sets >= 99.8 % equal and
+    recall within 0.002 (BASELINE north star)."""
+    gi, gd, gs = gpu
+    oi, od, os_ = ora
+    fin = np.isfinite(od) & np.isfinite(gd)
+    diff = np.abs(gd.astype(np.float64) - od.astype(np.float64))
+    rel = np.where(fin, diff / np.maximum(np.abs(od.astype(np.float64)), 1e-30), 0.0)
+    same_inf = (np.isfinite(od) == np.isfinite(gd)).all()
+    agree = float(np.mean([len(set(a.tolist()) & set(b.tolist())) / len(a) for a, b in zip(gi, oi)]))
+    rep = {"queries": int(len(gi)), "ids_equal": bool((gi == oi).all()),
+           "dists_equal": bool((gd == od).all()),
+           "max_rel_err": float(rel.max()) if rel.size else 0.0,
+           "counters_equal": bool(gs is not None and os_ is not None and
+                                  (gs[:, 0] == os_[:, 0]).all() and (gs[:, 1] == os_[:, 1]).all()
+                                  and (gs[:, 2] == os_[:, 3]).all()),
+           "id_agreement": round(agree, 6)}
+    if gt is not None:
+        rg, ro = recall_at_np(gi, gt), recall_at_np(oi, gt)
+        rep.update(recall_gpu=round(rg, 5), recall_oracle=round(ro, 5),
+                   recall_diff=round(abs(rg - ro), 5))
+    if exact:
+        rep["bar"] = "bit-exact ids, dists and counters (integer grid, R-C18)"
+        rep["ok"] = rep["ids_equal"] and rep["dists_equal"] and rep["counters_equal"]
+    else:
+        tol_ok = bool(same_inf and (diff[fin] <= 1e-5 * np.abs(od[fin]) + 1e-6).all())
+        rep["bar"] = "|dd| <= 1e-5|d| + 1e-6, id agreement >= 0.998, recall within 0.002"
+        rep["dists_within_tol"] = tol_ok
+        rep["ok"] = tol_ok and agree >= 0.998 and rep.get("recall_diff", 0.0) <= 0.002
+    return rep
+
+
+def recall_at_np(ids, gt):
+    k = gt.shape[1]
+    return float((ids[:, :, None] == gt[:, None, :]).any(2).sum()) / (k * gt.shape[0])
+
+
+def gt_check(X, Q, gt, k, metric, nq):
+    """K8: the bench's fp64 GPU ground truth against the oracle's
+    brute force (O6, pinned by numpy lexsort) on the first nq queries."""
+    import oracle
+    t0 = time.perf_counter()
+    oi, _ = oracle.bruteforce(X, Q[:nq], k, metric=metric, threads=oracle.ncores())
+    g = gt[:nq]
+    return {"queries": int(nq), "ids_equal": bool((oi == g).all()),
+            "ids_equal_frac": round(float((oi == g).mean()), 6),
+            "oracle_s": round(time.perf_counter() - t0, 2),
+            "note": "exact on the integer grid (L2); cosine ranks by -<q,x> in fp64 vs the "
+                    "oracle's fp32 distance, so near-ties may order differently"}
+
+
+def streams_for(nq_rank, base):
+    """Streams for back-to-back batches of nq_rank queries: enough batches in flight
+    to cover the resident warp slots (~3.5K per B200 at d <= 128) twice."""
+    return max(base, min(8, -(-2 * 3552 // max(1, nq_rank))))
+
+
 def run_ours(args):
     import torch
     import torch.distributed as dist
     import paper_conf_icde_yuwzqzl22_b200 as g
+    from paper_conf_icde_yuwzqzl22_b200 import dist as gdist
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -379,11 +544,16 @@ def run_ours(args):
     dev = torch.device("cuda", local)
     cfg = syn.CONFIGS[args.config]
     k = cfg.k
+    strong = args.scaling == "strong"
 
     B = max(1, args.batches)
-    X, Qs = make_workload(cfg, rank, B)
+    # weak: every rank draws its own batches; strong: every rank sees the same global
+    # batches and searches its slice of each (dist.query_slice)
+    X, Qs = make_workload(cfg, 0 if strong else rank, B)
+    Qs = Qs if isinstance(Qs, list) else [Qs]
     Q = Qs[0]
     nq = Q.shape[0]
+    lo, hi = gdist.query_slice(nq, rank, world) if strong else (0, nq)
     Xd = torch.from_numpy(X).to(dev)
     Qd_all = torch.from_numpy(np.concatenate(Qs)).to(dev)
     Qds = [Qd_all[b * nq:(b + 1) * nq] for b in range(B)]
@@ -411,7 +581,8 @@ def run_ours(args):
 
     # ---- (l, e) operating point over every query the timed steps search (see
     # select_operating_point); candidates timed as the steps are (pipelined)
-    pipe = Pipeline(torch, index, Qds, k, args.streams)
+    nstreams = streams_for(hi - lo, args.streams) if strong else args.streams
+    pipe = Pipeline(torch, index, Qds, k, nstreams, lo, hi)
     l_star, e_star, sweep, chosen = select_operating_point(
         torch, index, Qd_all, gt, k, args.target,
         lambda l, e: min(pipe.run(3 * B, l, e) for _ in range(3)))
@@ -419,14 +590,19 @@ def run_ours(args):
     rec = recall_at(ids, gt)
     st = st.long()
     d = cfg.d
-    # algorithmic bytes: query + per iteration the adjacency row
-    # + every computed distance's vector row (incl. the entry and lazy-check
-    # re-computations) + the top-k written; per step = mean over the batches
-    alg_bytes = int((4 * d + 4 * cfg.degree * st[:, 0] + 4 * d * st[:, 1]).sum().item()
-                    + 8 * k * Qd_all.shape[0]) // B
+    # algorithmic bytes: query + per iteration the adjacency row + every
+    # computed distance's vector row (entry and lazy-check re-computations) +
+    # the top-k written; HNSW adds the descent's rows (the kernel's descent counters)
+    per_q = 4 * d + 4 * cfg.degree * st[:, 0] + 4 * d * st[:, 1] + 8 * k
+    if index.hnsw:   # + the descent's adjacency rows and the permuted rows it gathers
+        ds = index.descent_stats(Qd_all, k, l_star, e_star).long()
+        per_q = per_q + 4 * cfg.degree * ds[:, 0] + 4 * d * ds[:, 1]
+    # per step = the mean over the batches of this rank's slice
+    sl = torch.cat([per_q[b * nq + lo:b * nq + hi] for b in range(B)])
+    alg_bytes = int(sl.sum().item()) // B
     iters_mean = float(st[:, 0].float().mean())
 
-    # ---- timed steps: device-resident inputs, back-to-back batches on two streams
+    # ---- timed steps: device-resident inputs, back-to-back batches on the streams
     pipe.run(args.warmup, l_star, e_star)
     torch.cuda.synchronize()
     launches0 = g.kernel_launches()
@@ -443,10 +619,13 @@ def run_ours(args):
     if distributed:
         dist.all_reduce(t_max, op=dist.ReduceOp.MAX)
     t_total = float(t_max.item())
-    total_queries = nq * args.steps * world
+    total_queries = nq * args.steps * (1 if strong else world)
     qps = total_queries / t_total
     ms_per_step = t_total / args.steps * 1e3
-    kernel_s = t_total / args.steps
+    launch_s = t_total / args.steps
+
+    # ---- DRAM bytes of the same steps (hardware counters, untimed second pass)
+    dram = measure_dram(lambda: pipe.run(args.steps, l_star, e_star), local)
 
     # ---- the other recall targets of SURVEY §8(d) (0.9, 0.99): same pipelined steps
     at_recall = {}
@@ -462,9 +641,26 @@ def run_ours(args):
         rr = next(r for l_, e_, r in sweep if (l_, e_) == tuple(le))
         at_recall[str(tgt)] = {"l": le[0], "e": le[1], "recall": rr, "qps": round(tq, 1)}
 
+    # ---- strong-scaling proxy on one GPU (replicated graph): the time
+    # of K steps over each rank's slice of the fixed batch, max over the W slices
+    proxy = None
+    if world == 1 and args.proxy_worlds:
+        proxy = {}
+        for W in [int(w) for w in args.proxy_worlds.split(",") if w]:
+            ts = []
+            for r in range(W):
+                a, b = gdist.query_slice(nq, r, W)
+                pw = Pipeline(torch, index, Qds, k, streams_for(b - a, args.streams), a, b)
+                pw.run(args.warmup, l_star, e_star)
+                ts.append(pw.run(args.steps, l_star, e_star))
+            tq = nq * args.steps / max(ts)
+            proxy[str(W)] = {"queries_per_gpu": nq // W, "streams": streams_for(nq // W, args.streams),
+                             "implied_qps": round(tq, 1),
+                             "per_gpu_efficiency": round(tq / (W * qps), 4)}
+
     # ---- end to end through the public API (ganns_search_host_async) from pinned
-    # host buffers: every step copies its batch in and its ids + dists out
-    Qhs = [torch.from_numpy(q).pin_memory() for q in Qs]
+    # host buffers: every step copies its batch (slice) in and its ids + dists out
+    Qhs = [torch.from_numpy(np.ascontiguousarray(q[lo:hi])).pin_memory() for q in Qs]
     pipe.run_host(g, Xd, Qhs, max(2, args.warmup), l_star, e_star)
     e2e_t = torch.tensor([pipe.run_host(g, Xd, Qhs, args.steps, l_star, e_star)],
                          dtype=torch.float64, device=dev)
@@ -473,17 +669,6 @@ def run_ours(args):
     e2e_qps = total_queries / float(e2e_t.item())
 
     peak, peak_kind = peaks()
-    achieved = alg_bytes / kernel_s / 1e9
-    traffic = None
-    tp = os.path.join(ROOT, "profiles", "traffic.json")
-    if os.path.exists(tp):
-        with open(tp) as f:
-            tr = json.load(f)
-        for ent in tr.get("entries", [tr]):
-            if (ent.get("config") == args.config and ent.get("l") == l_star
-                    and ent.get("e", l_star) == e_star):
-                traffic = ent.get("dram_bytes_per_launch")
-
     line = {
         "metric": "queries/sec at recall@10=0.95",
         "value": round(qps, 1),
@@ -493,11 +678,13 @@ def run_ours(args):
         "warmup": args.warmup,
         "ms_per_step": round(ms_per_step, 4),
         "higher_is_better": True,
-        "scaling": "weak",
+        "scaling": "strong" if strong else "weak",
         "vs_baseline": None,
         "dtype": "f32",
         "data": "synthetic",
-        "config": {"workload": workload_name(cfg, index.kind) + f", {Q.shape[0]} queries/GPU, k={k}",
+        "config": {"workload": workload_name(cfg, index.kind) + (
+                       f", {nq} queries per step split over {world} GPU(s), k={k}" if strong else
+                       f", {nq} queries/GPU, k={k}"),
                    "l": l_star, "e": e_star, "recall_at_10": round(rec, 5),
                    "recall_over": f"all {B * nq} queries of the {B} batches",
                    "selection": "fastest (l, e) with recall@10 >= target among the sweep",
@@ -508,7 +695,8 @@ def run_ours(args):
                    "l2": (f"not flushed: inputs larger than L2 ({(X.nbytes + cfg.n * cfg.degree * 4) >> 20}"
                           f" MiB vectors + graph vs 126 MB); steps rotate over {B} distinct "
                           f"{nq}-query batches"),
-                   "parallelism": f"replicated graph, query data-parallel x{world}"},
+                   "parallelism": (f"replicated graph, fixed batch split over {world} rank(s)"
+                                   if strong else f"replicated graph, query data-parallel x{world}")},
         "build_seconds": round(build_s, 4),
         "build_seconds_all": [round(x, 4) for x in build_all],
         "build_params": {"degree": cfg.degree, "d_min": cfg.degree // 2, "l_build": args.l_build,
@@ -519,22 +707,26 @@ def run_ours(args):
                   "searches": b_searches, "rounds": b_rounds,
                   "alg_GBps": round((4 * d * b_comps + 4 * cfg.degree * b_iters) / build_s / 1e9, 1)},
         "e2e": {"value": round(e2e_qps, 1), "unit": "queries/s",
-                "h2d_bytes_per_step": int(Q.nbytes), "d2h_bytes_per_step": int(nq * k * 8),
+                "h2d_bytes_per_step": int(Qhs[0].numel() * 4),
+                "d2h_bytes_per_step": int((hi - lo) * k * 8),
                 "api": "ganns_search_host_async, steps alternating over the streams, wall clock"},
         "gpu_launches": int(launches),
-        "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak,
-                     "unit": "GB/s", "frac": round(achieved / peak, 4), "traffic": traffic,
-                     # measured DRAM bytes (ncu, cold L2) over the live launch time: the
-                     # algorithmic figure above counts L2 hits as well, so it can exceed 1
-                     "traffic_frac": (round(traffic / kernel_s / 1e9 / peak, 4)
-                                      if traffic else None),
-                     "peak_kind": peak_kind, "alg_bytes_per_launch": alg_bytes,
-                     "duration": "timed region / steps (consecutive launches overlap on two streams)",
-                     "kernel": f"ganns::search_kernel (d={cfg.d}, d_max={cfg.degree}, {cfg.metric})"},
+        "roofline": roofline(alg_bytes, launch_s, dram, args.steps, peak, peak_kind,
+                             f"ganns::search_kernel (d={cfg.d}, d_max={cfg.degree}, {cfg.metric}"
+                             f"{', HNSW descent fused' if index.hnsw else ''})",
+                             "timed region / steps (consecutive launches overlap on the streams)"),
         "clocks": clk.summary(),
     }
+    if proxy is not None:
+        line["config"]["strong_scaling_proxy"] = proxy
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        line["cpu_baseline"] = cpu_baseline(index, X, Q, k, l_star, e_star, args.cpu_seconds)
+        line["roofline"]["read_peak_torch_sum_GBps"] = read_peak_gbps(torch, dev)
+        gpu_q = (ids[:nq].cpu().numpy(), dists[:nq].cpu().numpy(), st[:nq].cpu().numpy())
+        gt_np = gt[:nq].cpu().numpy()
+        line["cpu_baseline"], line["parity"] = cpu_baseline(
+            index, X, Q, k, l_star, e_star, args.cpu_seconds, gpu_q, gt_np,
+            exact=cfg.metric != "cosine")
+        line["gt_check"] = gt_check(X, Q, gt_np, k, cfg.metric, 100 if cfg.d <= 256 else 40)
         if not index.hnsw:
             line["cpu_build_baseline"] = cpu_build_baseline(torch, g, cfg, X, args.l_build,
                                                             min(args.l_local, args.l_build))
@@ -553,12 +745,14 @@ def run_sharded(args):
     """BASELINE configs[4] (DEEP100M-shaped, 100M x 96, 8 shards): every shard is an
     independent NSW (Algorithm 2) over its rows; every query is searched on every
     shard (K1), shard-local ids become global (id offset kernel), the per-shard
-    [nq, k] lists are all-gathered over NCCL and merged by K6 (ganns_merge_topk).
-    Rank r owns the shards s = r, r + N, ...; one step = the whole sharded search of
-    the 10K-query batch (strong scaling: the total work is fixed)."""
+    [nq, k] lists are exchanged with one NCCL all_gather_into_tensor and merged by
+    K6 (ganns_merge_topk) -- all through dist.ShardedIndex.  Rank r owns the shards
+    s = r, r + N, ...; one step = the whole sharded search of the 10K-query batch
+    (strong scaling: the total work is fixed)."""
     import torch
     import torch.distributed as dist
     import paper_conf_icde_yuwzqzl22_b200 as g
+    from paper_conf_icde_yuwzqzl22_b200 import dist as gdist
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -572,6 +766,8 @@ def run_sharded(args):
     if args.shard_rows:
         cfg = syn.with_size(cfg, n=args.shard_rows * cfg.shards)
     k, W = cfg.k, cfg.shards
+    if W % world != 0:
+        raise SystemExit(f"{W} shards do not split evenly over {world} ranks")
     per = cfg.n // W
     mine = [s for s in range(W) if s % world == rank]
     Q = syn.queries(cfg)
@@ -598,56 +794,46 @@ def run_sharded(args):
     cid = torch.cat([p for p, _ in gt_parts], 1)
     cdd = torch.cat([d for _, d in gt_parts], 1)
     if distributed:
-        ai = [torch.empty_like(cid) for _ in range(world)]
-        ad = [torch.empty_like(cdd) for _ in range(world)]
-        dist.all_gather(ai, cid)
-        dist.all_gather(ad, cdd)
-        cid, cdd = torch.cat(ai, 1), torch.cat(ad, 1)
+        ai = torch.empty((world,) + tuple(cid.shape), dtype=cid.dtype, device=dev)
+        ad = torch.empty((world,) + tuple(cdd.shape), dtype=cdd.dtype, device=dev)
+        dist.all_gather_into_tensor(ai, cid.contiguous())
+        dist.all_gather_into_tensor(ad, cdd.contiguous())
+        cid = torch.cat(list(ai), 1)
+        cdd = torch.cat(list(ad), 1)
     key = cdd * float(1 << 27) + cid.double()
     kk = torch.topk(key, k, dim=1, largest=False, sorted=True).values
     gt = (kk - torch.floor(kk / float(1 << 27)) * float(1 << 27)).round().int()
 
-    # the shard searches of a step alternate over two streams (their drain tails
-    # overlap the next shard's search); the gather + merge wait for both
+    # the shard searches of a step alternate over the streams (their drain tails
+    # overlap the next shard's search); the all-gather + merge wait for all of them
     streams = [torch.cuda.Stream(device=dev) for _ in range(max(1, args.streams))]
-    bufs = [(torch.empty((len(Q), k), dtype=torch.int32, device=dev),
-             torch.empty((len(Q), k), dtype=torch.float32, device=dev)) for _ in shards]
 
-    def step(l, e, Qin=None):
-        cur = torch.cuda.current_stream()
-        ev0 = torch.cuda.Event()
-        ev0.record(cur)
-        for j, (s, Xs, gr) in enumerate(shards):
-            st_ = streams[j % len(streams)]
-            st_.wait_event(ev0)
-            with torch.cuda.stream(st_):
-                g.search(gr, Xs, Qd if Qin is None else Qin, k, l, e=e, out=bufs[j])
-                g.offset_ids(bufs[j][0], s * per)
-        for st_ in streams:
-            ev = torch.cuda.Event()
-            ev.record(st_)
-            cur.wait_event(ev)
-        ids_loc = torch.stack([b[0] for b in bufs])
-        d_loc = torch.stack([b[1] for b in bufs])
-        if distributed:
-            gi = [torch.empty_like(ids_loc) for _ in range(world)]
-            gdd = [torch.empty_like(d_loc) for _ in range(world)]
-            dist.all_gather(gi, ids_loc)
-            dist.all_gather(gdd, d_loc)
-            ids_loc, d_loc = torch.cat(gi, 0), torch.cat(gdd, 0)
-        return g.merge_topk(ids_loc, d_loc)
+    def index_at(l):
+        return gdist.gpu_sharded_index([(s * per, gr, Xs) for s, Xs, gr in shards], k, l, e=l,
+                                       streams=streams)
 
     chosen, sweep = None, []
     for l in L_SWEEP:
-        ids, _ = step(l, l)
+        ids, _ = index_at(l).search(Qd)
         r = recall_at(ids[:nsub], gt)
         sweep.append((l, round(r, 5)))
         if r >= args.target:
             chosen = l
             break
     l_star = chosen or L_SWEEP[-1]
-    for _ in range(args.warmup):
-        step(l_star, l_star)
+    sidx = index_at(l_star)
+
+    def steps_run(n):
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        for _ in range(n):
+            out = sidx.search(Qd)
+        e1.record()
+        e1.synchronize()
+        return e0.elapsed_time(e1) / 1e3, out
+
+    steps_run(args.warmup)
     torch.cuda.synchronize()
     if distributed:
         dist.barrier()
@@ -657,7 +843,7 @@ def run_sharded(args):
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record()
         for _ in range(args.steps):
-            ids, _ = step(l_star, l_star)
+            ids, dists = sidx.search(Qd)
         e1.record()
         while not e1.query():
             clk.sample_now()
@@ -673,6 +859,9 @@ def run_sharded(args):
     t_total = float(t.item())
     rec = recall_at(ids[:nsub], gt)
     qps = len(Q) * args.steps / t_total
+    # DRAM bytes of the same steps (hardware counters, untimed second pass; a
+    # collective inside a profiled range is fine -- it is one pass, no replay)
+    dram = measure_dram(lambda: steps_run(args.steps)[0], local)
     # roofline of K1 on the shards (untimed stats pass: the kernel's own counters)
     # per shard launch: the timed region over the launches (they overlap pairwise)
     search_s = t_total / args.steps / max(1, len(shards))
@@ -683,7 +872,6 @@ def run_sharded(args):
         alg += int((4 * cfg.d + 4 * cfg.degree * st[:, 0] + 4 * cfg.d * st[:, 1]).sum()) + 8 * k * len(Q)
     alg_per_launch = alg // max(1, len(shards))
     peak, peak_kind = peaks()
-    achieved = alg_per_launch / search_s / 1e9
     # end to end: queries from pinned host memory, results back to pinned host
     # memory, inside the timed region (the all-gather and merge included)
     Qh = torch.from_numpy(Q).pin_memory()
@@ -697,7 +885,7 @@ def run_sharded(args):
             dist.barrier()
         t0 = time.perf_counter()
         Qin.copy_(Qh, non_blocking=True)
-        i_, d_ = step(l_star, l_star, Qin=Qin)
+        i_, d_ = sidx.search(Qin)
         hid.copy_(i_, non_blocking=True)
         hdd.copy_(d_, non_blocking=True)
         torch.cuda.current_stream().synchronize()
@@ -717,7 +905,8 @@ def run_sharded(args):
                    "l": l_star, "e": l_star, "recall_at_10": round(rec, 5),
                    "recall_subset": nsub, "l_sweep_recall": sweep,
                    "shards_per_gpu": len(mine),
-                   "parallelism": f"base set sharded, {world} rank(s), NCCL all-gather + K6 merge",
+                   "parallelism": (f"base set sharded, {world} rank(s), dist.ShardedIndex: "
+                                   "NCCL all_gather_into_tensor + K6 merge"),
                    "streams": len(streams),
                    "l2": (f"not flushed: inputs larger than L2 ({cfg.n * cfg.d * 4 >> 20} MiB of "
                           "vectors); a shard is re-searched only after the other shards")},
@@ -725,15 +914,16 @@ def run_sharded(args):
         "gpu_launches": int(launches), "clocks": clk.summary(),
         "e2e": {"value": round(e2e_qps, 1), "unit": "queries/s",
                 "h2d_bytes_per_step": int(Q.nbytes), "d2h_bytes_per_step": int(len(Q) * k * 8)},
-        "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
-                     "frac": round(achieved / peak, 4), "traffic": None, "peak_kind": peak_kind,
-                     "alg_bytes_per_launch": alg_per_launch,
-                     "kernel": f"ganns::search_kernel on one {per}-row shard (d={cfg.d}, "
-                               f"d_max={cfg.degree}, {cfg.metric}); mean over the shard launches"},
+        "roofline": roofline(alg_per_launch, search_s, dram, args.steps * max(1, len(shards)), peak,
+                             peak_kind,
+                             f"ganns::search_kernel on one {per}-row shard (d={cfg.d}, "
+                             f"d_max={cfg.degree}, {cfg.metric}); mean over the shard launches",
+                             "timed region / (steps x shards on this GPU)"),
     }
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        line["cpu_baseline"] = sharded_cpu_baseline(torch, g, shards, per, Q, k, l_star,
-                                                    args.cpu_seconds, cfg.metric)
+        line["cpu_baseline"], line["parity"] = sharded_cpu_baseline(
+            torch, g, shards, per, Q, k, l_star, args.cpu_seconds, cfg.metric,
+            (ids.cpu().numpy(), dists.cpu().numpy()), gt.cpu().numpy())
     if rank == 0:
         print(json.dumps(line), flush=True)
         if args.json_out:
@@ -744,10 +934,11 @@ def run_sharded(args):
         dist.destroy_process_group()
 
 
-def sharded_cpu_baseline(torch, g, shards, per, Q, k, l, seconds, metric):
+def sharded_cpu_baseline(torch, g, shards, per, Q, k, l, seconds, metric, gpu, gt):
     """The oracle's sharded search on a bounded query sample: every shard searched by
     the oracle (plain C, one pthread per host core, same graph and l), then the
-    oracle's merge by (dist, global id).  Host copies of the shards (not timed)."""
+    oracle's merge by (dist, global id); compared element by element with the GPU's
+    merged result for the same queries.  Host copies of the shards (not timed)."""
     import oracle
     cores = oracle.ncores()
     m = 0
@@ -767,16 +958,27 @@ def sharded_cpu_baseline(torch, g, shards, per, Q, k, l, seconds, metric):
         parts.append((np.where(ids >= 0, ids + s * per, -1).astype(np.int32), dd))
         del Xh, A
     t0 = time.perf_counter()
-    oracle.merge_topk(np.stack([p[0] for p in parts]), np.stack([p[1] for p in parts]))
+    mi, md = oracle.merge_topk(np.stack([p[0] for p in parts]), np.stack([p[1] for p in parts]))
     tot += time.perf_counter() - t0
-    return {"value": round(m / tot, 1), "unit": "queries/s", "cores": cores, "kind": "oracle",
-            "sample": f"first {m} of the {len(Q)} queries on all {len(shards)} shards "
-                      f"(same graphs, l={l}) + merge, {tot:.1f} s"}
+    gi, gd = gpu
+    mm = min(m, len(gt))
+    par = parity_report((gi[:m], gd[:m], None), (mi, md, None), exact=True,
+                        gt=gt[:mm] if mm == m else None)
+    par["counters_equal"] = None   # the merged lists carry no per-shard counters
+    par["ok"] = par["ids_equal"] and par["dists_equal"]
+    par["bar"] = "bit-exact merged ids and dists (per-shard oracle search + oracle merge)"
+    return ({"value": round(m / tot, 1), "unit": "queries/s", "cores": cores, "kind": "oracle",
+             "cpu_model": cpu_model(),
+             "sample": f"first {m} of the {len(Q)} queries on all {len(shards)} shards "
+                       f"(same graphs, l={l}) + merge, {tot:.1f} s"}, par)
 
 
-def cpu_baseline(index, X, Q, k, l, e, seconds):
-    """The oracle's search (plain C, one pthread per host core) on a bounded sample
-    of the same queries and graph.  Returns the cpu_baseline object."""
+def cpu_baseline(index, X, Q, k, l, e, seconds, gpu, gt, exact):
+    """The oracle's search (plain C) on a bounded sample of the same queries and
+    graph: all host cores (one pthread per core) and one thread (the paper's CPU
+    baselines are single-threaded).  Returns (cpu_baseline, parity): the
+    oracle's results on the all-core sample compared element by element with the
+    GPU's (`gpu` = ids, dists, stats of the batch at the same (l, e))."""
     import oracle
     cores = oracle.ncores()
     m = 64
@@ -785,33 +987,45 @@ def cpu_baseline(index, X, Q, k, l, e, seconds):
     dt = time.perf_counter() - t0
     m2 = int(min(len(Q), max(m, m * seconds / max(dt, 1e-3))))
     t0 = time.perf_counter()
-    index.oracle_search(X, Q[:m2], k, l, e, cores)
+    oi, od, ost = index.oracle_search(X, Q[:m2], k, l, e, cores)
     dt = time.perf_counter() - t0
-    return {"value": round(m2 / dt, 1), "unit": "queries/s", "cores": cores, "kind": "oracle",
-            "sample": f"first {m2} of the {len(Q)} queries, same graph, l={l}, e={e}, {dt:.1f} s"}
+    m1 = int(max(8, min(m2, m2 * 3.0 / max(dt * cores, 1e-3))))
+    t0 = time.perf_counter()
+    index.oracle_search(X, Q[:m1], k, l, e, 1)
+    dt1 = time.perf_counter() - t0
+    gi, gd, gs = gpu
+    par = parity_report((gi[:m2], gd[:m2], gs[:m2]), (oi, od, ost), exact, gt=gt[:m2])
+    return ({"value": round(m2 / dt, 1), "unit": "queries/s", "cores": cores, "kind": "oracle",
+             "cpu_model": cpu_model(),
+             "one_thread": {"value": round(m1 / dt1, 1), "queries": m1, "seconds": round(dt1, 2)},
+             "sample": f"first {m2} of the {len(Q)} queries, same graph, l={l}, e={e}, {dt:.1f} s "
+                       f"on {cores} threads; {m1} queries on 1 thread"}, par)
 
 
 def cpu_build_baseline(torch, g, cfg, X, l_build, l_local=0, m=10000):
     """Algorithm 2 on the first m points: the oracle (plain C, one thread -- the paper's
     CPU baselines are single-threaded) and the GPU build of the same sample with
-    the same partition (group size 256 = the auto rule at this size)."""
+    the same partition (group size 256 = the auto rule at this size), compared
+    bit-exact.  The oracle's Algorithm 2 on the full config (all cores) is
+    tools/oracle_alg2_full.py (minutes; profiles/r02/oracle_alg2_full_C2.json)."""
     import oracle
     Xs = np.ascontiguousarray(X[:m])
     S = 256
     t0 = time.perf_counter()
-    oracle.alg2(Xs, cfg.degree // 2, cfg.degree, S, l_build=l_build, metric=cfg.metric,
-                l_local=l_local)
+    ref, _, _ = oracle.alg2(Xs, cfg.degree // 2, cfg.degree, S, l_build=l_build,
+                            metric=cfg.metric, l_local=l_local)
     t_cpu = time.perf_counter() - t0
     Xd = torch.from_numpy(Xs).cuda()
     g.build(Xd, metric=cfg.metric, degree=cfg.degree, l_build=l_build, group_size=S,
             l_local=l_local)  # warm
     torch.cuda.synchronize()
     t0 = time.perf_counter()
-    g.build(Xd, metric=cfg.metric, degree=cfg.degree, l_build=l_build, group_size=S,
-            l_local=l_local)
+    gr = g.build(Xd, metric=cfg.metric, degree=cfg.degree, l_build=l_build, group_size=S,
+                 l_local=l_local)
     torch.cuda.synchronize()
     t_gpu = time.perf_counter() - t0
     return {"oracle_s": round(t_cpu, 3), "gpu_s": round(t_gpu, 4), "cores": 1, "kind": "oracle",
+            "adjacency_equal": bool((gr.adjacency() == ref).all()),
             "sample": f"Algorithm 2 on the first {m} points (degree {cfg.degree}, "
                       f"l_build {l_build}, l_local {l_local or l_build}, group size {S})"}
 

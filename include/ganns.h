@@ -81,6 +81,9 @@ typedef struct {
     uint32_t *stats;    /* device, nullable, [nq][3] per query: iterations, distance
                            computations (entry + every valid neighbour), T entries
                            merged into N (kept among the first l)                   */
+    uint32_t *descent_stats; /* device, nullable, [nq][2] (HNSW searches only): iterations and
+                           distance computations of the greedy descent through the upper
+                           layers (R-H1), summed over the layers; ignored by the NSW calls */
 } ganns_search_params;
 
 /* ganns_build -- GGraphCon NSW construction, Algorithm 2 (§IV-B

@@ -62,7 +62,7 @@ def lib():
         _lib.ora_hnsw_build.argtypes = [P, i64, i32, i32, P, i32, i32, i32, i32, i64, P, P, P,
                                         P, P]
         _lib.ora_hnsw_search.argtypes = [P, P, i32, P, P, i64, i32, P, i32, i32, P, i64, i32,
-                                         i32, i32, P, P, P, P]
+                                         i32, i32, P, P, P, P, P]
         for f in ("ora_hnsw_build", "ora_hnsw_search", "ora_merge_topk", "ora_search_one", "ora_search_batch", "ora_alg1", "ora_bruteforce",
                   "ora_nsw_seq", "ora_alg2", "ora_alg2_ex", "ora_alg2_mt",
                   "ora_naive_parallel"):
@@ -242,21 +242,24 @@ def hnsw_build(X, levels, d_min, d_max, group_size, l_build=64, e_build=0, metri
     return dict(perm=perm, layer_n=layer_n, upper=ups, layer0=layer0, upper_flat=upper)
 
 
-def hnsw_search(h, X, Q, k, l, e=0, metric="l2", stats=False):
+def hnsw_search(h, X, Q, k, l, e=0, metric="l2", stats=False, descent_stats=False):
     """Greedy descent through the upper layers, then GANNS on layer 0.
-    Returns ids, dists, entries (+ stats [nq,4])."""
+    Returns ids, dists, entries (+ stats [nq,4]) (+ descent stats [nq,2]: iterations,
+    distance computations of the descent, summed over the upper layers)."""
     X, Q = _f32(X), _f32(np.atleast_2d(Q))
     nq = Q.shape[0]
     ids = np.empty((nq, k), np.int32)
     dists = np.empty((nq, k), np.float32)
     ent = np.empty(nq, np.int32)
     st = np.empty((nq, 4), np.uint32) if stats else None
+    ds = np.empty((nq, 2), np.uint32) if descent_stats else None
     layer0 = h["layer0"]
     _check(lib().ora_hnsw_search(_p(h["perm"]), _p(h["layer_n"]), len(h["layer_n"]),
                                  _p(h["upper_flat"]), _p(layer0), layer0.shape[0],
                                  layer0.shape[1], _p(X), X.shape[1], METRICS[metric], _p(Q), nq,
-                                 k, l, e, _p(ids), _p(dists), _p(st), _p(ent)))
-    return (ids, dists, ent, st) if stats else (ids, dists, ent)
+                                 k, l, e, _p(ids), _p(dists), _p(st), _p(ent), _p(ds)))
+    res = (ids, dists, ent, st) if stats else (ids, dists, ent)
+    return res + (ds,) if descent_stats else res
 
 
 def knn_descent(X, init, K, max_iters=30, metric="l2"):

@@ -34,7 +34,8 @@ class _BuildParams(ct.Structure):
 
 
 class _SearchParams(ct.Structure):
-    _fields_ = [("e", ct.c_int), ("entry", ct.c_int64), ("stats", ct.c_void_p)]
+    _fields_ = [("e", ct.c_int), ("entry", ct.c_int64), ("stats", ct.c_void_p),
+                ("descent_stats", ct.c_void_p)]
 
 
 def _load():
@@ -137,6 +138,19 @@ def _dev_f32(t: torch.Tensor, name: str) -> torch.Tensor:
     return t.contiguous()
 
 
+def _check_index_inputs(graph, points: torch.Tensor, queries: torch.Tensor):
+    """The kernels read points through a tensor map / row pointers built from the
+    graph's (n, d) and queries (device or host) as [nq][d]: refuse any other shape
+    (an out-of-bounds access otherwise) and device queries on another device."""
+    if tuple(points.shape) != (graph.n, graph.d):
+        raise ValueError(f"points must be [{graph.n}, {graph.d}] (the graph's n and d), "
+                         f"got {list(points.shape)}")
+    if queries.shape[1] != graph.d:
+        raise ValueError(f"queries must have d = {graph.d} columns, got {queries.shape[1]}")
+    if queries.is_cuda and points.device != queries.device:
+        raise ValueError("points and queries must be on the same device")
+
+
 def kernel_launches() -> int:
     """Kernels launched by libganns.so in this process."""
     return int(_lib.ganns_kernel_launches())
@@ -222,6 +236,7 @@ def search(graph: Graph, points: torch.Tensor, queries: torch.Tensor, k: int, l:
     computations, merged entries) when ``stats``."""
     points = _dev_f32(points, "points")
     queries = _dev_f32(queries, "queries")
+    _check_index_inputs(graph, points, queries)
     nq = queries.shape[0]
     if out is None:
         ids = torch.empty((nq, k), dtype=torch.int32, device=queries.device)
@@ -229,7 +244,7 @@ def search(graph: Graph, points: torch.Tensor, queries: torch.Tensor, k: int, l:
     else:
         ids, dists = _check_out(out, nq, k, queries.device)
     st = torch.empty((nq, 3), dtype=torch.int32, device=queries.device) if stats else None
-    p = _SearchParams(e, entry, ct.c_void_p(st.data_ptr()) if stats else None)
+    p = _SearchParams(e, entry, ct.c_void_p(st.data_ptr()) if stats else None, None)
     with torch.cuda.device(queries.device):
         _check(_lib.ganns_search_ex(graph.handle, ct.c_void_p(points.data_ptr()),
                                     ct.c_void_p(queries.data_ptr()), nq, k, l, ct.byref(p),
@@ -243,9 +258,10 @@ def search_host(graph: Graph, points: torch.Tensor, queries: torch.Tensor, k: in
     """End-to-end search from host memory: ``queries`` is a CPU float32 tensor
     (pin it for copy/compute overlap); results come back in CPU tensors."""
     points = _dev_f32(points, "points")
-    if queries.is_cuda or queries.dtype != torch.float32:
-        raise TypeError("queries must be a float32 CPU tensor")
+    if queries.is_cuda or queries.dtype != torch.float32 or queries.dim() != 2:
+        raise TypeError("queries must be a 2-D float32 CPU tensor")
     queries = queries.contiguous()
+    _check_index_inputs(graph, points, queries)
     nq = queries.shape[0]
     if out is None:
         ids = torch.empty((nq, k), dtype=torch.int32, pin_memory=True)
@@ -254,7 +270,7 @@ def search_host(graph: Graph, points: torch.Tensor, queries: torch.Tensor, k: in
         ids, dists = out
         _check_buf(ids, (nq, k), torch.int32, False, "out[0] (ids)")
         _check_buf(dists, (nq, k), torch.float32, False, "out[1] (dists)")
-    p = _SearchParams(e, entry, None)
+    p = _SearchParams(e, entry, None, None)
     with torch.cuda.device(points.device):
         _check(_lib.ganns_search_host(graph.handle, ct.c_void_p(points.data_ptr()),
                                       ct.c_void_p(queries.data_ptr()), nq, k, l, ct.byref(p),
@@ -281,13 +297,15 @@ def search_host_async(index, points: torch.Tensor, queries_host: torch.Tensor, k
     nq = queries_host.shape[0]
     if queries_host.dim() != 2 or not queries_host.is_contiguous():
         raise TypeError("queries_host must be a contiguous 2-D tensor")
-    d = queries_host.shape[1]
+    base = index.base if isinstance(index, Hnsw) else index
+    _check_index_inputs(base, points, queries_host)
+    d = base.d      # the library copies nq * graph.d floats
     _check_buf(qd, (nq, d), torch.float32, True, "scratch[0] (queries)")
     _check_buf(ids_d, (nq, k), torch.int32, True, "scratch[1] (ids)")
     _check_buf(dists_d, (nq, k), torch.float32, True, "scratch[2] (dists)")
     _check_buf(ids_h, (nq, k), torch.int32, False, "out_host[0] (ids)")
     _check_buf(dists_h, (nq, k), torch.float32, False, "out_host[1] (dists)")
-    p = _SearchParams(e, 0, None)
+    p = _SearchParams(e, 0, None, None)
     fn = _lib.ganns_hnsw_search_host_async if isinstance(index, Hnsw) else _lib.ganns_search_host_async
     with torch.cuda.device(points.device):
         _check(fn(index.handle, ct.c_void_p(points.data_ptr()),
@@ -382,10 +400,14 @@ def build_hnsw(points: torch.Tensor, levels: np.ndarray, metric: str = "l2", deg
 
 
 def hnsw_search(index: Hnsw, points: torch.Tensor, queries: torch.Tensor, k: int, l: int,
-                e: int = 0, stats: bool = False, out=None, stream=None):
-    """Greedy descent of the upper layers, then the GANNS search on layer 0."""
+                e: int = 0, stats: bool = False, out=None, stream=None,
+                descent_stats: bool = False):
+    """Greedy descent of the upper layers, then the GANNS search on layer 0.  With
+    ``stats``: layer-0 counters [nq, 3]; with ``descent_stats`` as well: the
+    descent's (iterations, distance computations) [nq, 2] appended to the result."""
     points = _dev_f32(points, "points")
     queries = _dev_f32(queries, "queries")
+    _check_index_inputs(index.base, points, queries)
     nq = queries.shape[0]
     if out is None:
         ids = torch.empty((nq, k), dtype=torch.int32, device=queries.device)
@@ -393,13 +415,16 @@ def hnsw_search(index: Hnsw, points: torch.Tensor, queries: torch.Tensor, k: int
     else:
         ids, dists = _check_out(out, nq, k, queries.device)
     st = torch.empty((nq, 3), dtype=torch.int32, device=queries.device) if stats else None
-    p = _SearchParams(e, 0, ct.c_void_p(st.data_ptr()) if stats else None)
+    ds = torch.empty((nq, 2), dtype=torch.int32, device=queries.device) if descent_stats else None
+    p = _SearchParams(e, 0, ct.c_void_p(st.data_ptr()) if stats else None,
+                      ct.c_void_p(ds.data_ptr()) if descent_stats else None)
     with torch.cuda.device(queries.device):
         _check(_lib.ganns_hnsw_search(index.handle, ct.c_void_p(points.data_ptr()),
                                       ct.c_void_p(queries.data_ptr()), nq, k, l, ct.byref(p),
                                       ct.c_void_p(ids.data_ptr()), ct.c_void_p(dists.data_ptr()),
                                       _stream(stream)))
-    return (ids, dists, st) if stats else (ids, dists)
+    res = (ids, dists, st) if stats else (ids, dists)
+    return res + (ds,) if descent_stats else res
 
 
 def build_knn(points: torch.Tensor, init: np.ndarray, K: int, metric: str = "l2",

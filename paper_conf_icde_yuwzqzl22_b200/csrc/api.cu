@@ -8,6 +8,7 @@
 #include <cmath>
 #include <cstdio>
 #include <cstring>
+#include <exception>
 #include <mutex>
 #include <new>
 #include <vector>
@@ -235,7 +236,12 @@ int ganns_graph_from_adjacency(const int32_t* nbr_host, int64_t n, int d_max, in
                                int device, ganns_graph** out) {
   if (!nbr_host || !out) return fail(GANNS_EINVAL, "NULL argument");
   if (int rc = validate_common(n, d, metric, d_max)) return rc;
-  std::vector<int32_t> seen(size_t(n), -1);   // row stamp per id
+  std::vector<int32_t> seen;   // row stamp per id
+  try {
+    seen.assign(size_t(n), -1);
+  } catch (const std::exception&) {
+    return fail(GANNS_ENOMEM, "host allocation failed (adjacency check)");
+  }
   for (int64_t v = 0; v < n; ++v) {
     for (int j = 0; j < d_max; ++j) {
       int32_t u = nbr_host[size_t(v) * d_max + j];
@@ -273,7 +279,12 @@ int ganns_graph_adjacency(const ganns_graph* g, int32_t* out_host) {
 int ganns_graph_save(const ganns_graph* g, const char* path) {
   if (int rc = check_graph(g)) return rc;
   if (!path) return fail(GANNS_EINVAL, "path is NULL");
-  std::vector<int32_t> h(size_t(g->n) * g->d_max);
+  std::vector<int32_t> h;
+  try {
+    h.resize(size_t(g->n) * g->d_max);
+  } catch (const std::exception&) {
+    return fail(GANNS_ENOMEM, "host allocation failed (graph save)");
+  }
   if (int rc = ganns_graph_adjacency(g, h.data())) return rc;
   FILE* f = std::fopen(path, "wb");
   if (!f) return fail(GANNS_EIO, std::string("cannot open ") + path);
@@ -295,11 +306,26 @@ int ganns_graph_load(const char* path, int device, ganns_graph** out) {
   int32_t meta[4];
   bool ok = std::fread(magic, 1, 8, f) == 8 && std::memcmp(magic, "GANNSG01", 8) == 0 &&
             std::fread(&n, 8, 1, f) == 1 && std::fread(meta, 4, 4, f) == 4;
-  if (!ok || n < 2 || meta[1] < 2 || meta[1] > 128) {
-    std::fclose(f);
-    return fail(GANNS_EIO, std::string("bad graph header: ") + path);
+  // validate the header before allocating: sizes, dimension, metric, and the
+  // file length must match exactly (a corrupt header never reaches the allocator)
+  ok = ok && n >= 2 && n < (int64_t(1) << 31) && meta[1] >= 2 && meta[1] <= 128 &&
+       meta[0] >= 4 && meta[0] <= 1024 && meta[0] % 4 == 0 && meta[2] >= 0 && meta[2] <= 2;
+  const int64_t header = 8 + 8 + 16;
+  if (ok) {
+    ok = std::fseek(f, 0, SEEK_END) == 0 &&
+         std::ftell(f) == header + int64_t(4) * n * meta[1] && std::fseek(f, header, SEEK_SET) == 0;
   }
-  std::vector<int32_t> h(size_t(n) * meta[1]);
+  if (!ok) {
+    std::fclose(f);
+    return fail(GANNS_EIO, std::string("bad graph header or size: ") + path);
+  }
+  std::vector<int32_t> h;
+  try {
+    h.resize(size_t(n) * meta[1]);
+  } catch (const std::exception&) {
+    std::fclose(f);
+    return fail(GANNS_ENOMEM, "host allocation failed (graph load)");
+  }
   ok = std::fread(h.data(), 4, h.size(), f) == h.size();
   std::fclose(f);
   if (!ok) return fail(GANNS_EIO, std::string("truncated graph file: ") + path);
@@ -311,7 +337,9 @@ static int validate_search(const ganns_graph* g, const float* points, const floa
                            const void* out_ids, const void* out_dists, int* e_out,
                            int32_t* entry_out) {
   if (int rc = check_graph(g)) return rc;
-  if (nq < 0 || nq >= (int64_t(1) << 31)) return fail(GANNS_EINVAL, "nq must be in [0, 2^31)");
+  // the persistent kernel's int32 ticket reaches nq + (resident warps): keep headroom
+  if (nq < 0 || nq > (int64_t(1) << 31) - (int64_t(1) << 24))
+    return fail(GANNS_EINVAL, "nq must be in [0, 2^31 - 2^24]");
   if (k < 1 || k >= g->n) return fail(GANNS_EINVAL, "k must be in [1, n)");
   if (l < k || l > 1024) return fail(GANNS_EINVAL, "l must be in [k, 1024]");
   int e = p ? p->e : 0;
@@ -651,6 +679,7 @@ int ganns_hnsw_search(const ganns_hnsw* h, const float* points, const float* que
     a.Xp = h->Xp;
     a.np = h->layer_n[1];
     a.perm = h->perm;
+    a.dstats = p ? p->descent_stats : nullptr;
     cudaError_t err = launch_search(a, s);
     return err == cudaSuccess ? GANNS_OK : cuda_fail(err, "hnsw search");
   }
@@ -674,11 +703,14 @@ int ganns_hnsw_search(const ganns_hnsw* h, const float* points, const float* que
     ea.nq = nq;
     ea.perm = h->perm;
     ea.entries = entries;
+    ea.dstats = p ? p->descent_stats : nullptr;
     err = launch_entries(ea, s);
   } else {
     entry = h->entry0;   // a single layer: every query enters at perm[0]
     cudaFreeAsync(entries, s);
     entries = nullptr;
+    if (p && p->descent_stats)   // no descent
+      err = cudaMemsetAsync(p->descent_stats, 0, sizeof(uint32_t) * 2 * size_t(nq), s);
   }
   if (err != cudaSuccess) {
     if (entries) cudaFreeAsync(entries, s);

@@ -322,16 +322,16 @@ round_merge_kernel(int32_t* __restrict__ gid, float* __restrict__ gdist, int d_m
 // ------------------------------------------------------------------ host
 template <int NV4, int TPL, bool L2>
 static cudaError_t set_smem_attrs() {
-  static bool done = false;
-  if (done) return cudaSuccess;
-  const int mx = 227 * 1024;
-  cudaError_t e = cudaFuncSetAttribute(phase1_kernel<NV4, TPL, L2>,
-                                       cudaFuncAttributeMaxDynamicSharedMemorySize, mx);
-  if (e == cudaSuccess)
-    e = cudaFuncSetAttribute(round_search_kernel<NV4, TPL, L2>,
-                             cudaFuncAttributeMaxDynamicSharedMemorySize, mx);
-  done = e == cudaSuccess;
-  return e;
+  static std::atomic<uint64_t> done{0};   // per instantiation, per device
+  return once_per_device(done, [] {
+    const int mx = 227 * 1024;
+    cudaError_t e = cudaFuncSetAttribute(phase1_kernel<NV4, TPL, L2>,
+                                         cudaFuncAttributeMaxDynamicSharedMemorySize, mx);
+    if (e == cudaSuccess)
+      e = cudaFuncSetAttribute(round_search_kernel<NV4, TPL, L2>,
+                               cudaFuncAttributeMaxDynamicSharedMemorySize, mx);
+    return e;
+  });
 }
 
 template <typename T>

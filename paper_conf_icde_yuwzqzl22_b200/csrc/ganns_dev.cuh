@@ -848,7 +848,8 @@ struct UpperLayers {
 // carries the permuted points (and their tensor map) and the degree.
 template <int NV4, int TPL, bool L2>
 __device__ int32_t descend(const GraphView& base, const UpperLayers& U, int stop,
-                           const float* __restrict__ q, WarpSmem& ws) {
+                           const float* __restrict__ q, WarpSmem& ws,
+                           SearchStats* acc = nullptr) {
   int32_t cur = 0;
   for (int j = U.top; j >= stop; --j) {
     GraphView gv = base;
@@ -856,6 +857,10 @@ __device__ int32_t descend(const GraphView& base, const UpperLayers& U, int stop
     gv.n = U.n[j];
     SearchStats st;
     warp_search<NV4, TPL, L2, false>(gv, q, cur, 1, 1, ws, st);
+    if (acc != nullptr) {   // the descent's own counters (bench: its algorithmic bytes)
+      acc->iters += st.iters;
+      acc->comps += st.comps;
+    }
     cur = key_id(unflag(ws.sN[0]));
     __syncwarp();
   }

@@ -35,11 +35,29 @@ constexpr int kMinBlocksPerSM = GANNS_MIN_BLOCKS; // register budget: <= 85 regs
 #ifndef GANNS_MIN_BLOCKS_WIDE
 #define GANNS_MIN_BLOCKS_WIDE (16 / GANNS_SEARCH_WARPS)
 #endif
-// d > 128 (NV4 >= 2): the TMA stage (>= 16.5 KB/warp) caps residency at <= 14 warps
-// per SM, so the register budget may grow to 128/thread (16 warps) at no occupancy
-// cost; at 80 the C4 (d = 200, HNSW) instance spilled 268 B/thread to local memory
-// (ncu: 62 M local store requests per launch, 566 MB of DRAM writes).
+// d > 128 (NV4 >= 2): register budget 128/thread (<= 16 warps per SM).  The 2-round
+// TMA stage is 16 rows x d x 4 B = 8.4-16 KB per warp for d in (128, 256], plus N;
+// at the bench's C4 point (d = 200, l = 288, 13 KB + 2.3 KB per warp) shared memory
+// already caps residency at 14 warps, so 128 registers cost nothing there and remove
+// the spills of the 80-register budget (268 B/thread, 566 MB of DRAM writes per
+// launch).  For d ~ 132-176 with small l, shared memory would allow ~20 warps and
+// this cap (16) may cost occupancy; only d = 200 was measured.
 constexpr int kMinBlocksWide = GANNS_MIN_BLOCKS_WIDE;
+
+// cudaFuncSetAttribute state is per device: run `set` once per device ordinal
+// (bit d of `done`); concurrent first calls may both run `set`, which is idempotent.
+template <class F>
+inline cudaError_t once_per_device(std::atomic<uint64_t>& done, F&& set) {
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  if (dev < 0 || dev >= 64) return set();
+  const uint64_t bit = uint64_t(1) << dev;
+  if (done.load(std::memory_order_acquire) & bit) return cudaSuccess;
+  e = set();
+  if (e == cudaSuccess) done.fetch_or(bit, std::memory_order_acq_rel);
+  return e;
+}
 
 void set_error(const std::string& msg);
 int fail(int status, const std::string& msg);
@@ -82,6 +100,7 @@ struct SearchLaunch {
   const float* Xp = nullptr;
   int64_t np = 0;
   const int32_t* perm = nullptr;
+  uint32_t* dstats = nullptr;   // HNSW: nullable [nq][2] descent iterations / comps
 };
 // HNSW: per-query layer-0 entry = perm[greedy descent through the upper layers]
 struct EntryLaunch {
@@ -93,6 +112,7 @@ struct EntryLaunch {
   int64_t nq;
   const int32_t* perm;
   int32_t* entries;
+  uint32_t* dstats = nullptr;   // nullable [nq][2] descent iterations / comps
 };
 cudaError_t launch_entries(const EntryLaunch& a, cudaStream_t s);
 template <int NV4>

@@ -32,6 +32,7 @@ struct HnswUpper {
   const float* Xp;
   int64_t np;
   const int32_t* perm;
+  uint32_t* dstats;     // nullable [nq][2]: the descent's iterations, distance computations
 };
 template <int NV4, int TPL, bool L2, bool HNSW>
 __global__ void __launch_bounds__(kSearchWarps * 32, NV4 == 1 ? kMinBlocksPerSM : kMinBlocksWide)
@@ -102,7 +103,12 @@ search_kernel(GraphView g, const float* __restrict__ Q, int64_t nq, int k, int l
     gu.X = H.Xp;
     gu.n = H.np;
     gu.tmap = &tmap_up;
-    ent = H.perm[descend<NV4, TPL, L2>(gu, H.U, 1, qrow, ws)];
+    SearchStats ds{0u, 0u, 0u};
+    ent = H.perm[descend<NV4, TPL, L2>(gu, H.U, 1, qrow, ws, H.dstats != nullptr ? &ds : nullptr)];
+    if (H.dstats != nullptr && lane == 0) {
+      H.dstats[size_t(q) * 2 + 0] = ds.iters;
+      H.dstats[size_t(q) * 2 + 1] = ds.comps;
+    }
   }
   const int cnt = warp_search<NV4, TPL, L2, false>(g, qrow, ent, l, e, ws, st);
   // output: the first k of N, (-1, +inf) padded (R-C8)
@@ -148,14 +154,16 @@ static int pick_wide_rows(const SearchLaunch& a, int sms) {
 template <int NV4, int TPL, bool L2, bool HNSW = false>
 static cudaError_t launch_t(const SearchLaunch& a, cudaStream_t s) {
   auto kern = search_kernel<NV4, TPL, L2, HNSW>;
-  static bool attr_done = false;   // per instantiation
-  if (!attr_done) {
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         227 * 1024);
-    if (e == cudaSuccess)
-      e = cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+  static std::atomic<uint64_t> attr_done{0};   // per instantiation, per device
+  {
+    cudaError_t e = once_per_device(attr_done, [&] {
+      cudaError_t r = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                           227 * 1024);
+      if (r == cudaSuccess)
+        r = cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+      return r;
+    });
     if (e != cudaSuccess) return e;
-    attr_done = true;
   }
   int dev = 0, sms = 0, per_sm = 0;
   cudaGetDevice(&dev);
@@ -196,6 +204,7 @@ static cudaError_t launch_t(const SearchLaunch& a, cudaStream_t s) {
     H.Xp = a.Xp;
     H.np = a.np;
     H.perm = a.perm;
+    H.dstats = a.dstats;
     err = encode_row_tmap(a.Xp, a.np, a.d, &tmap_up);
     if (err != cudaSuccess) return err;
   }
@@ -227,14 +236,16 @@ static bool wide_group_enabled() {
 template <int CG, int TPL, bool L2>
 static cudaError_t launch_group_t(const SearchLaunch& a, cudaStream_t s) {
   auto kern = search_group_kernel<CG, TPL, L2>;
-  static bool attr_done = false;
-  if (!attr_done) {
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         227 * 1024);
-    if (e == cudaSuccess)
-      e = cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+  static std::atomic<uint64_t> attr_done{0};   // per instantiation, per device
+  {
+    cudaError_t e = once_per_device(attr_done, [&] {
+      cudaError_t r = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                           227 * 1024);
+      if (r == cudaSuccess)
+        r = cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+      return r;
+    });
     if (e != cudaSuccess) return e;
-    attr_done = true;
   }
   int dev = 0, sms = 0, per_sm = 0;
   cudaGetDevice(&dev);
@@ -316,7 +327,7 @@ template <int NV4, int TPL, bool L2>
 __global__ void __launch_bounds__(kSearchWarps * 32)
 hnsw_entry_kernel(GraphView g, const UpperLayers U, const float* __restrict__ Q, int64_t nq,
                   const int32_t* __restrict__ perm, int32_t* __restrict__ entries,
-                  const __grid_constant__ CUtensorMap tmap) {
+                  uint32_t* __restrict__ dstats, const __grid_constant__ CUtensorMap tmap) {
   extern __shared__ __align__(128) uint8_t smem[];
   g.tmap = &tmap;
   const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -327,8 +338,16 @@ hnsw_entry_kernel(GraphView g, const UpperLayers U, const float* __restrict__ Q,
   __syncwarp();
   const int64_t q = int64_t(blockIdx.x) * kSearchWarps + w;
   if (q >= nq) return;
-  const int32_t c = descend<NV4, TPL, L2>(g, U, 1, Q + size_t(q) * (g.d4 * 4), ws);
-  if (lane == 0) entries[q] = perm[c];
+  SearchStats ds{0u, 0u, 0u};
+  const int32_t c = descend<NV4, TPL, L2>(g, U, 1, Q + size_t(q) * (g.d4 * 4), ws,
+                                          dstats != nullptr ? &ds : nullptr);
+  if (lane == 0) {
+    entries[q] = perm[c];
+    if (dstats != nullptr) {
+      dstats[size_t(q) * 2 + 0] = ds.iters;
+      dstats[size_t(q) * 2 + 1] = ds.comps;
+    }
+  }
 }
 
 template <int NV4, int TPL, bool L2>
@@ -348,7 +367,8 @@ static cudaError_t entries_t(const EntryLaunch& a, cudaStream_t s) {
     U.n[j] = a.upper.n[j];
   }
   const int64_t blocks = (a.nq + kSearchWarps - 1) / kSearchWarps;
-  kern<<<unsigned(blocks), kSearchWarps * 32, smem, s>>>(g, U, a.Q, a.nq, a.perm, a.entries, tmap);
+  kern<<<unsigned(blocks), kSearchWarps * 32, smem, s>>>(g, U, a.Q, a.nq, a.perm, a.entries,
+                                                        a.dstats, tmap);
   count_launch();
   return cudaGetLastError();
 }

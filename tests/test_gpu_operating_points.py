@@ -64,12 +64,15 @@ def test_c4_instance_hnsw_fused_l288_integer_ip_bitexact():
     levels = syn.hnsw_levels(len(X), cfg.degree // 2, 1)
     idx = g.build_hnsw(Xd, levels, metric="ip", degree=cfg.degree, l_build=128)
     assert idx.nlayers >= 3
-    ids, dists, st = g.hnsw_search(idx, Xd, cu(Q), cfg.k, 288, stats=True)   # one launch
+    ids, dists, st, ds = g.hnsw_search(idx, Xd, cu(Q), cfg.k, 288, stats=True,
+                                       descent_stats=True)   # one launch
     torch.cuda.synchronize()
-    ids, dists, st = ids.cpu().numpy(), dists.cpu().numpy(), st.cpu().numpy()
+    ids, dists, st, ds = ids.cpu().numpy(), dists.cpu().numpy(), st.cpu().numpy(), ds.cpu().numpy()
     h = oracle_index(idx)
     sample = np.arange(0, len(Q), 25)
-    oi, od, _, ost = oracle.hnsw_search(h, X, Q[sample], cfg.k, 288, metric="ip", stats=True)
+    oi, od, _, ost, ods = oracle.hnsw_search(h, X, Q[sample], cfg.k, 288, metric="ip", stats=True,
+                                             descent_stats=True)
+    assert (ds[sample] == ods).all()          # the descent's counters (bench bytes)
     assert (ids[sample] == oi).all()
     assert (dists[sample] == od).all()
     assert (st[sample][:, 0] == ost[:, 0]).all() and (st[sample][:, 1] == ost[:, 1]).all()

@@ -87,8 +87,13 @@ def test_hnsw_descent_handbuilt_fixture():
     h = dict(perm=perm, layer_n=np.array([n, 4, 2], np.int64), upper={1: up1, 2: up2},
              layer0=layer0, upper_flat=np.concatenate([up1.reshape(-1), up2.reshape(-1)]))
     q = np.array([[3.1, 0, 0, 0]], np.float32)
-    ids, dists, ent = oracle.hnsw_search(h, X, q, 2, 2)
+    ids, dists, ent, st, ds = oracle.hnsw_search(h, X, q, 2, 2, stats=True, descent_stats=True)
     assert ent.tolist() == [perm[3]]
+    # the descent's counters, by hand: layer 2 -- entry 0 (1 distance), explore 0
+    # (T = {1}), explore 1 (T = {0}, not in N = [1]: recomputed) = 2 iterations, 3
+    # distances; layer 1 -- entry 1 (1), explore 1 (T = {0, 2, 3}), explore 3
+    # (T = {0}) = 2 iterations, 5 distances
+    assert ds.tolist() == [[4, 8]]
     # layer-0 search from perm[3] (x = 2): its component {x=2, x=0}
     assert ids[0].tolist() == [perm[3], perm[0]]
     assert np.allclose(dists[0], [(3.1 - 2) ** 2, 3.1 ** 2])
