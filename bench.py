@@ -51,7 +51,7 @@ def parse():
     ap.add_argument("--target", type=float, default=0.95)
     ap.add_argument("--l-build", type=int, default=128,
                     help="candidate-list length of the build searches (P:222: 32/64/128)")
-    ap.add_argument("--l-local", type=int, default=64,
+    ap.add_argument("--l-local", type=int, default=32,
                     help="list length of the Phase-1 (local graph) build searches, <= l_build "
                          "(R-C13; 0 = l_build); not used by the HNSW config")
     ap.add_argument("--no-cpu-baseline", action="store_true")

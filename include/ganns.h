@@ -102,6 +102,62 @@ typedef struct {
 GANNS_API int ganns_build(const float *points, int64_t n, int d, int metric, int degree,
                 const ganns_build_params *p, void *stream, ganns_graph **out);
 
+/* ---------------------------------------------------------------- staged build
+ * Algorithm 2 one step at a time, for a construction split over several working
+ * units (the paper's Remarks: "each working unit ... builds one local
+ * graph" and the searches of an iteration are independent).  Every rank holds
+ * the same points and a full replica of the graph state; a rank runs Phase 1 for
+ * its share of the groups and the Phase-2 searches for its share of each round's
+ * vertices; the caller exchanges the results (ganns_build_rows, the F blocks)
+ * and every rank applies the same round, so the replicas stay bit-identical to
+ * ganns_build with the same parameters (python: dist.build_distributed).
+ *
+ * ganns_build_begin  -- validate (exactly as ganns_build) and allocate the state
+ *   and the graph rows on the current device; returns the state in *out.
+ *   p->max_rounds / stop_after_phase1 / stats are ignored (the caller drives the
+ *   rounds; ganns_build_finish returns the counters).
+ * ganns_build_info   -- group size s (R-C14), number of groups t + 1,
+ *   d_min, d_max.  Group g holds vertices [g*s, min((g+1)*s, n)).
+ * ganns_build_phase1 -- Alg. 2 lines 2-8 for groups [g0, g1) (a group's
+ *   insertions touch only its own rows); async on `stream`.
+ * ganns_build_rows   -- copy the build-form rows of vertices [v0, v1) out of
+ *   (to_state = 0) or into (to_state = 1) the state: device buffers ids / dists
+ *   [v1-v0][d_max] (row-major, -1 / +inf padded) and pids / pdists [v1-v0][d_min]
+ *   (N').  Importing whole groups marks them ready for Phase 2.
+ * ganns_build_round_search -- Alg. 2 lines 10-17 of round i (1 <= i <= t) for
+ *   the vertices [v0, v1) of P_i: writes each v's new forward row F (the first
+ *   d_min of Search(G_0, v) u v.N' by (dist, id), R-C16) to f_ids / f_dists
+ *   (device, [v1-v0][d_min], -1 / +inf padded).  Requires Phase 1 of groups
+ *   0..i and rounds 1..i-1 applied.  Reads the state only.
+ * ganns_build_round_apply -- the rest of round i from the F of ALL of P_i
+ *   (f_ids / f_dists [|P_i|][d_min], in vertex order): rows of P_i <- F (R-C15),
+ *   E from F (line 17), GatherScatter and the per-vertex merges (lines 19-22).
+ *   Rounds must be applied in order 1, 2, ..., t.
+ * ganns_build_finish -- syncs `stream`; *out receives the graph (same as
+ *   ganns_build's), stats (nullable, host [4]) the build counters (search
+ *   iterations, distance computations, searches run on THIS rank, rounds); the
+ *   state is freed.
+ * ganns_build_abort  -- frees a state and its graph (NULL is a no-op).
+ * Errors: GANNS_EINVAL for out-of-range groups / vertices / rounds, rounds out of
+ *   order, or a round before its groups are ready; otherwise as ganns_build. */
+typedef struct ganns_build_state ganns_build_state;
+GANNS_API int ganns_build_begin(const float *points, int64_t n, int d, int metric, int degree,
+                                const ganns_build_params *p, void *stream,
+                                ganns_build_state **out);
+GANNS_API int ganns_build_info(const ganns_build_state *s, int64_t *group_size,
+                               int64_t *ngroups, int *d_min, int *d_max);
+GANNS_API int ganns_build_phase1(ganns_build_state *s, int64_t g0, int64_t g1, void *stream);
+GANNS_API int ganns_build_rows(ganns_build_state *s, int64_t v0, int64_t v1, int32_t *ids,
+                               float *dists, int32_t *pids, float *pdists, int to_state,
+                               void *stream);
+GANNS_API int ganns_build_round_search(ganns_build_state *s, int64_t i, int64_t v0, int64_t v1,
+                                       int32_t *f_ids, float *f_dists, void *stream);
+GANNS_API int ganns_build_round_apply(ganns_build_state *s, int64_t i, const int32_t *f_ids,
+                                      const float *f_dists, void *stream);
+GANNS_API int ganns_build_finish(ganns_build_state *s, void *stream, uint64_t *stats,
+                                 ganns_graph **out);
+GANNS_API void ganns_build_abort(ganns_build_state *s);
+
 /* ganns_search -- batched GANNS search (§III-B): for each query,
  * the k approximate nearest neighbours (Def. 1) found with a
  * candidate array of length l (lazy update) and the lazy check.

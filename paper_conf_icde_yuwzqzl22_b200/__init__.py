@@ -69,6 +69,13 @@ def _load():
         "ganns_hnsw_base": [P, ct.POINTER(P)],
         "ganns_build_knn": [P, i64, i32, i32, i32, P, i32, P, ct.POINTER(P), ct.POINTER(i32),
                             ct.POINTER(i64)],
+        "ganns_build_begin": [P, i64, i32, i32, i32, ct.POINTER(_BuildParams), P, ct.POINTER(P)],
+        "ganns_build_info": [P, ct.POINTER(i64), ct.POINTER(i64), ct.POINTER(i32), ct.POINTER(i32)],
+        "ganns_build_phase1": [P, i64, i64, P],
+        "ganns_build_rows": [P, i64, i64, P, P, P, P, i32, P],
+        "ganns_build_round_search": [P, i64, i64, i64, P, P, P],
+        "ganns_build_round_apply": [P, i64, P, P, P],
+        "ganns_build_finish": [P, P, P, ct.POINTER(P)],
     }
     for name, args in sig.items():
         f = getattr(lib, name)
@@ -78,6 +85,8 @@ def _load():
     lib.ganns_graph_free.restype = None
     lib.ganns_hnsw_free.argtypes = [P]
     lib.ganns_hnsw_free.restype = None
+    lib.ganns_build_abort.argtypes = [P]
+    lib.ganns_build_abort.restype = None
     lib.ganns_last_error.argtypes = []
     lib.ganns_last_error.restype = ct.c_char_p
     lib.ganns_kernel_launches.argtypes = []
@@ -95,7 +104,9 @@ ABI_SYMBOLS = ("ganns_build", "ganns_search", "ganns_search_ex", "ganns_search_h
                "ganns_graph_save", "ganns_graph_load", "ganns_graph_free", "ganns_last_error",
                "ganns_kernel_launches", "ganns_build_hnsw", "ganns_hnsw_search",
                "ganns_hnsw_info", "ganns_hnsw_layer", "ganns_hnsw_perm", "ganns_hnsw_base",
-               "ganns_hnsw_free", "ganns_build_knn")
+               "ganns_hnsw_free", "ganns_build_knn", "ganns_build_begin", "ganns_build_info",
+               "ganns_build_phase1", "ganns_build_rows", "ganns_build_round_search",
+               "ganns_build_round_apply", "ganns_build_finish", "ganns_build_abort")
 
 
 def lib():
@@ -227,6 +238,102 @@ def build(points: torch.Tensor, metric: str = "l2", degree: int = 32, d_min: int
     g = Graph(h)
     g.build_stats = tuple(int(x) for x in st)
     return g
+
+
+class StagedBuild:
+    """Algorithm 2 one step at a time (ganns_build_begin ... ganns_build_finish; the
+    multi-GPU construction of dist.build_distributed).  Same parameters as build().
+    Every method enqueues on `stream` (default: the current stream)."""
+
+    def __init__(self, points: torch.Tensor, metric: str = "l2", degree: int = 32, d_min: int = 0,
+                 l_build: int = 0, e_build: int = 0, group_size: int = 0, l_local: int = 0,
+                 stream=None):
+        self.points = _dev_f32(points, "points")
+        self.device = self.points.device
+        self.stream = stream
+        self.n, self.d = self.points.shape
+        p = _BuildParams(d_min, l_build, e_build, group_size, 0, 0, None, l_local)
+        h = ct.c_void_p()
+        with torch.cuda.device(self.device):
+            _check(_lib.ganns_build_begin(ct.c_void_p(self.points.data_ptr()), self.n, self.d,
+                                          METRICS[metric], degree, ct.byref(p),
+                                          _stream(stream), ct.byref(h)))
+        self._h = h
+        s, t, dm, dx = ct.c_int64(), ct.c_int64(), ct.c_int(), ct.c_int()
+        _check(_lib.ganns_build_info(h, ct.byref(s), ct.byref(t), ct.byref(dm), ct.byref(dx)))
+        self.group_size, self.ngroups, self.d_min, self.d_max = s.value, t.value, dm.value, dx.value
+
+    def _p(self, t):
+        return ct.c_void_p(t.data_ptr())
+
+    def info(self):
+        return self.group_size, self.ngroups, self.d_min, self.d_max
+
+    def group_rows(self, g0: int, g1: int):
+        """Vertex range [v0, v1) of groups [g0, g1)."""
+        return min(g0 * self.group_size, self.n), min(g1 * self.group_size, self.n)
+
+    def phase1(self, g0: int, g1: int):
+        with torch.cuda.device(self.device):
+            _check(_lib.ganns_build_phase1(self._h, g0, g1, _stream(self.stream)))
+
+    def export_rows(self, v0: int, v1: int):
+        """(ids [m, d_max], dists, pids [m, d_min], pdists) of vertices [v0, v1)."""
+        m = v1 - v0
+        kw = dict(device=self.device)
+        out = (torch.empty((m, self.d_max), dtype=torch.int32, **kw),
+               torch.empty((m, self.d_max), dtype=torch.float32, **kw),
+               torch.empty((m, self.d_min), dtype=torch.int32, **kw),
+               torch.empty((m, self.d_min), dtype=torch.float32, **kw))
+        with torch.cuda.device(self.device):
+            _check(_lib.ganns_build_rows(self._h, v0, v1, *(self._p(t) for t in out), 0,
+                                         _stream(self.stream)))
+        return out
+
+    def import_rows(self, v0: int, v1: int, rows):
+        m = v1 - v0
+        shapes = ((m, self.d_max), (m, self.d_max), (m, self.d_min), (m, self.d_min))
+        dts = (torch.int32, torch.float32, torch.int32, torch.float32)
+        for t, shp, dt, nm in zip(rows, shapes, dts, ("ids", "dists", "pids", "pdists")):
+            _check_buf(t, shp, dt, True, nm)
+        with torch.cuda.device(self.device):
+            _check(_lib.ganns_build_rows(self._h, v0, v1, *(self._p(t) for t in rows), 1,
+                                         _stream(self.stream)))
+
+    def round_search(self, i: int, v0: int, v1: int):
+        """New forward rows F of vertices [v0, v1) of P_i: (ids, dists) [v1-v0, d_min]."""
+        f = (torch.empty((v1 - v0, self.d_min), dtype=torch.int32, device=self.device),
+             torch.empty((v1 - v0, self.d_min), dtype=torch.float32, device=self.device))
+        with torch.cuda.device(self.device):
+            _check(_lib.ganns_build_round_search(self._h, i, v0, v1, self._p(f[0]), self._p(f[1]),
+                                                 _stream(self.stream)))
+        return f
+
+    def round_apply(self, i: int, f_ids: torch.Tensor, f_dists: torch.Tensor):
+        lo, hi = self.group_rows(i, i + 1)
+        _check_buf(f_ids, (hi - lo, self.d_min), torch.int32, True, "f_ids")
+        _check_buf(f_dists, (hi - lo, self.d_min), torch.float32, True, "f_dists")
+        with torch.cuda.device(self.device):
+            _check(_lib.ganns_build_round_apply(self._h, i, self._p(f_ids), self._p(f_dists),
+                                                _stream(self.stream)))
+
+    def finish(self) -> Graph:
+        st = (ct.c_uint64 * 4)()
+        h = ct.c_void_p()
+        with torch.cuda.device(self.device):
+            _check(_lib.ganns_build_finish(self._h, _stream(self.stream),
+                                           ct.cast(st, ct.POINTER(ct.c_uint64)), ct.byref(h)))
+        self._h = None
+        g = Graph(h)
+        g.build_stats = tuple(int(x) for x in st)
+        return g
+
+    def __del__(self):
+        try:
+            if self._h:
+                _lib.ganns_build_abort(self._h)
+        except Exception:
+            pass
 
 
 def search(graph: Graph, points: torch.Tensor, queries: torch.Tensor, k: int, l: int,

@@ -21,7 +21,8 @@ FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-fvisibility=hid
          "-I", os.path.join(ROOT, "include")] + os.environ.get("GANNS_NVCC_EXTRA", "").split()
 
 # (source, extra defines, object name)
-UNITS = [("api.cu", [], "api.o"), ("search.cu", [], "search.o"), ("knn.cu", [], "knn.o")] + \
+UNITS = [("api.cu", [], "api.o"), ("search.cu", [], "search.o"), ("knn.cu", [], "knn.o"),
+         ("build.cu", [], "build.o")] + \
         [("search_inst.cu", [f"-DGANNS_NV4={v}"], f"search_nv{v}.o") for v in (1, 2, 4, 8)] + \
         [("build_inst.cu", [f"-DGANNS_NV4={v}"], f"build_nv{v}.o") for v in (1, 2, 4, 8)]
 # GANNS_DEV=1: developer flavour with only the d <= 128 / d_max <= 32 / L2
@@ -30,6 +31,7 @@ UNITS = [("api.cu", [], "api.o"), ("search.cu", [], "search.o"), ("knn.cu", [], 
 DEV_UNITS = [("api.cu", ["-DGANNS_DEV_NV1"], "dev_api.o"),
              ("search.cu", ["-DGANNS_DEV_NV1"], "dev_search.o"),
              ("knn.cu", [], "dev_knn.o"),
+             ("build.cu", ["-DGANNS_DEV_NV1"], "dev_build.o"),
              ("search_inst.cu", ["-DGANNS_NV4=1", "-DGANNS_DEV_ONE"], "dev_search_nv1.o"),
              ("build_inst.cu", ["-DGANNS_NV4=1", "-DGANNS_DEV_ONE"], "dev_build_nv1.o")]
 FLAVOR = os.path.join(PKG, "libganns.flavor")

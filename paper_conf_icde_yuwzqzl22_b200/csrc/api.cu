@@ -124,17 +124,6 @@ int32_t* ticket_slot() {
   return g_tickets[dev] + (g_ticket_next.fetch_add(1) % kTicketSlots);
 }
 
-int run_build(BuildArgs& a, cudaStream_t s) {
-  switch (nv4_for(a.d)) {
-    case 1: return run_build_nv<1>(a, s);
-#ifndef GANNS_DEV_NV1
-    case 2: return run_build_nv<2>(a, s);
-    case 4: return run_build_nv<4>(a, s);
-    case 8: return run_build_nv<8>(a, s);
-#endif
-  }
-  return fail(GANNS_ENOTSUP, "unsupported dimension");
-}
 
 // H2D, search, D2H of one batch on `stream` (no sync); `search` enqueues the search
 // on the device copies.
@@ -465,9 +454,10 @@ int ganns_search_host_async(const ganns_graph* g, const float* points, const flo
                     });
 }
 
-int ganns_build(const float* points, int64_t n, int d, int metric, int degree,
-                const ganns_build_params* p, void* stream, ganns_graph** out) {
-  if (!points || !out) return fail(GANNS_EINVAL, "NULL argument");
+// Arguments of Algorithm 2 (validated; defaults applied) -> BuildArgs.
+static int build_args(const float* points, int64_t n, int d, int metric, int degree,
+                      const ganns_build_params* p, BuildArgs* out) {
+  if (!points) return fail(GANNS_EINVAL, "NULL argument");
   if (int rc = validate_common(n, d, metric, degree)) return rc;
   if (!aligned16(points)) return fail(GANNS_EINVAL, "points not 16-byte aligned");
   int d_min = p && p->d_min > 0 ? p->d_min : degree / 2;
@@ -480,12 +470,10 @@ int ganns_build(const float* points, int64_t n, int d, int metric, int degree,
   if (e_build < 1 || e_build > l_build) return fail(GANNS_EINVAL, "e_build must be in [1, l_build]");
   const int l_local = p && p->l_local > 0 ? p->l_local : l_build;
   if (l_local < d_min || l_local > l_build) return fail(GANNS_EINVAL, "l_local must be in [d_min, l_build]");
+  if (p && p->group_size < 0) return fail(GANNS_EINVAL, "group_size < 0");
   int64_t S = p && p->group_size > 0 ? p->group_size : 0;
   if (S == 0) S = auto_group_size(n);
   if (S > n) S = n;
-  if (p && p->group_size < 0) return fail(GANNS_EINVAL, "group_size < 0");
-  int rc = new_graph(n, d, degree, metric, out);
-  if (rc) return rc;
   BuildArgs a{};
   a.X = points;
   a.n = n;
@@ -499,6 +487,17 @@ int ganns_build(const float* points, int64_t n, int d, int metric, int degree,
   a.e_local = std::min(e_build, l_local);
   a.group_size = S;
   a.max_rounds = p ? (p->stop_after_phase1 ? 0 : (p->max_rounds > 0 ? p->max_rounds : -1)) : -1;
+  *out = a;
+  return GANNS_OK;
+}
+
+int ganns_build(const float* points, int64_t n, int d, int metric, int degree,
+                const ganns_build_params* p, void* stream, ganns_graph** out) {
+  if (!points || !out) return fail(GANNS_EINVAL, "NULL argument");
+  BuildArgs a{};
+  if (int rc = build_args(points, n, d, metric, degree, p, &a)) return rc;
+  int rc = new_graph(n, d, degree, metric, out);
+  if (rc) return rc;
   a.out_nbr = (*out)->nbr;
   rc = run_build(a, static_cast<cudaStream_t>(stream));
   if (rc) {
@@ -510,6 +509,157 @@ int ganns_build(const float* points, int64_t n, int d, int metric, int degree,
     for (int i = 0; i < 4; ++i) p->stats[i] = a.stats[i];
   return GANNS_OK;
 }
+
+// ------------------------------------------------ staged Algorithm 2 (NEXT-2)
+}  // extern "C"
+
+struct ganns_build_state {
+  ganns::BuildState st;
+  ganns_graph* graph = nullptr;   // the rows being built (becomes the result)
+  int64_t rounds_applied = 0;
+};
+
+namespace {
+int check_state(const ganns_build_state* s) {
+  if (!s || !s->graph || !s->st.phase1) return fail(GANNS_EINVAL, "build state is NULL or finished");
+  return GANNS_OK;
+}
+int64_t group_lo(const BuildState& st, int64_t g) { return std::min(g * st.S, st.a.n); }
+}  // namespace
+
+extern "C" {
+
+int ganns_build_begin(const float* points, int64_t n, int d, int metric, int degree,
+                      const ganns_build_params* p, void* stream, ganns_build_state** out) {
+  if (!points || !out) return fail(GANNS_EINVAL, "NULL argument");
+  BuildArgs a{};
+  if (int rc = build_args(points, n, d, metric, degree, p, &a)) return rc;
+  ganns_build_state* s = new (std::nothrow) ganns_build_state();
+  if (!s) return fail(GANNS_ENOMEM, "host allocation failed");
+  int rc = new_graph(n, d, degree, metric, &s->graph);
+  if (rc) {
+    delete s;
+    return rc;
+  }
+  a.out_nbr = s->graph->nbr;
+  s->st.a = a;
+  rc = build_begin(s->st, static_cast<cudaStream_t>(stream));
+  if (rc) {
+    ganns_build_abort(s);
+    return rc;
+  }
+  s->st.group_ready.assign(size_t(s->st.ngroups), 0);
+  *out = s;
+  return GANNS_OK;
+}
+
+int ganns_build_info(const ganns_build_state* s, int64_t* group_size, int64_t* ngroups,
+                     int* d_min, int* d_max) {
+  if (int rc = check_state(s)) return rc;
+  if (group_size) *group_size = s->st.S;
+  if (ngroups) *ngroups = s->st.ngroups;
+  if (d_min) *d_min = s->st.a.d_min;
+  if (d_max) *d_max = s->st.a.d_max;
+  return GANNS_OK;
+}
+
+int ganns_build_phase1(ganns_build_state* s, int64_t g0, int64_t g1, void* stream) {
+  if (int rc = check_state(s)) return rc;
+  BuildState& st = s->st;
+  if (g0 < 0 || g1 > st.ngroups || g0 > g1) return fail(GANNS_EINVAL, "groups must satisfy 0 <= g0 <= g1 <= ngroups");
+  if (s->rounds_applied > 0) return fail(GANNS_EINVAL, "Phase 1 after a Phase-2 round");
+  if (int rc = st.phase1(st, g0, g1, static_cast<cudaStream_t>(stream))) return rc;
+  for (int64_t g = g0; g < g1; ++g) st.group_ready[size_t(g)] = 1;
+  return GANNS_OK;
+}
+
+int ganns_build_rows(ganns_build_state* s, int64_t v0, int64_t v1, int32_t* ids, float* dists,
+                     int32_t* pids, float* pdists, int to_state, void* stream) {
+  if (int rc = check_state(s)) return rc;
+  BuildState& st = s->st;
+  if (v0 < 0 || v1 > st.a.n || v0 > v1) return fail(GANNS_EINVAL, "rows must satisfy 0 <= v0 <= v1 <= n");
+  if (v1 > v0 && (!ids || !dists || !pids || !pdists)) return fail(GANNS_EINVAL, "NULL buffer");
+  const size_t m = size_t(v1 - v0), dmax = size_t(st.a.d_max), dm = size_t(st.a.d_min);
+  const cudaMemcpyKind k = cudaMemcpyDeviceToDevice;
+  cudaStream_t cs = static_cast<cudaStream_t>(stream);
+  int32_t* gid = s->graph->nbr + size_t(v0) * dmax;
+  float* gd = st.gdist + size_t(v0) * dmax;
+  int32_t* gpi = st.gpid + size_t(v0) * dm;
+  float* gpd = st.gpd + size_t(v0) * dm;
+  cudaError_t e;
+  if (to_state) {
+    e = cudaMemcpyAsync(gid, ids, 4 * m * dmax, k, cs);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(gd, dists, 4 * m * dmax, k, cs);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(gpi, pids, 4 * m * dm, k, cs);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(gpd, pdists, 4 * m * dm, k, cs);
+  } else {
+    e = cudaMemcpyAsync(ids, gid, 4 * m * dmax, k, cs);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(dists, gd, 4 * m * dmax, k, cs);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(pids, gpi, 4 * m * dm, k, cs);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(pdists, gpd, 4 * m * dm, k, cs);
+  }
+  if (e != cudaSuccess) return cuda_fail(e, "ganns_build_rows");
+  if (to_state)   // whole groups covered by imported rows are ready for Phase 2
+    for (int64_t g = 0; g < st.ngroups; ++g)
+      if (group_lo(st, g) >= v0 && group_lo(st, g + 1) <= v1) st.group_ready[size_t(g)] = 1;
+  return GANNS_OK;
+}
+
+int ganns_build_round_search(ganns_build_state* s, int64_t i, int64_t v0, int64_t v1,
+                             int32_t* f_ids, float* f_dists, void* stream) {
+  if (int rc = check_state(s)) return rc;
+  BuildState& st = s->st;
+  if (i < 1 || i >= st.ngroups) return fail(GANNS_EINVAL, "round must be in [1, ngroups)");
+  if (i != s->rounds_applied + 1) return fail(GANNS_EINVAL, "rounds must be applied in order");
+  for (int64_t g = 0; g <= i; ++g)
+    if (!st.group_ready[size_t(g)]) return fail(GANNS_EINVAL, "Phase 1 of a group <= i is missing");
+  const int64_t lo = group_lo(st, i), hi = group_lo(st, i + 1);
+  if (v0 < lo || v1 > hi || v0 > v1) return fail(GANNS_EINVAL, "vertices must lie in P_i");
+  if (v1 > v0 && (!f_ids || !f_dists)) return fail(GANNS_EINVAL, "NULL buffer");
+  return st.round_search(st, i, v0, v1, f_ids, f_dists, static_cast<cudaStream_t>(stream));
+}
+
+int ganns_build_round_apply(ganns_build_state* s, int64_t i, const int32_t* f_ids,
+                            const float* f_dists, void* stream) {
+  if (int rc = check_state(s)) return rc;
+  BuildState& st = s->st;
+  if (i < 1 || i >= st.ngroups) return fail(GANNS_EINVAL, "round must be in [1, ngroups)");
+  if (i != s->rounds_applied + 1) return fail(GANNS_EINVAL, "rounds must be applied in order");
+  if (!f_ids || !f_dists) return fail(GANNS_EINVAL, "NULL buffer");
+  for (int64_t g = 0; g <= i; ++g)
+    if (!st.group_ready[size_t(g)]) return fail(GANNS_EINVAL, "Phase 1 of a group <= i is missing");
+  if (int rc = st.round_apply(st, i, f_ids, f_dists, static_cast<cudaStream_t>(stream))) return rc;
+  s->rounds_applied = i;
+  return GANNS_OK;
+}
+
+int ganns_build_finish(ganns_build_state* s, void* stream, uint64_t* stats, ganns_graph** out) {
+  if (int rc = check_state(s)) return rc;
+  if (!out) return fail(GANNS_EINVAL, "NULL argument");
+  cudaStream_t cs = static_cast<cudaStream_t>(stream);
+  unsigned long long hs[3];
+  cudaError_t e = cudaMemcpyAsync(hs, s->st.stats, sizeof(hs), cudaMemcpyDeviceToHost, cs);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(cs);
+  if (e != cudaSuccess) return cuda_fail(e, "ganns_build_finish");
+  if (stats) {
+    stats[0] = hs[0];
+    stats[1] = hs[1];
+    stats[2] = hs[2];
+    stats[3] = uint64_t(s->rounds_applied);
+  }
+  *out = s->graph;
+  s->graph = nullptr;
+  delete s;   // frees the scratch
+  return GANNS_OK;
+}
+
+void ganns_build_abort(ganns_build_state* s) {
+  if (!s) return;
+  if (s->graph) ganns_graph_free(s->graph);
+  s->graph = nullptr;
+  delete s;
+}
+
 
 // ---------------------------------------------------------------- HNSW
 }  // extern "C"

@@ -27,6 +27,7 @@
 // row ∪ segment, which does not depend on it -- the graph is bit-identical to
 // sorting E by (u, dist, v) (R-C17).
 #include "ganns_dev.cuh"
+#include "../../include/ganns.h"
 #include "ganns_internal.h"
 
 #ifndef GANNS_NV4
@@ -35,6 +36,7 @@
 
 #include <algorithm>
 #include <cmath>
+#include <new>
 #include <vector>
 
 namespace ganns {
@@ -117,13 +119,13 @@ __device__ __forceinline__ void add_stats(unsigned long long* st, const SearchSt
 // Phase 1: local graph construction (Alg. 2 lines 2-8).
 template <int NV4, int TPL, bool L2>
 __global__ void __launch_bounds__(kBuildWarps * 32)
-phase1_kernel(BuildDev B, int64_t group_size, int64_t ngroups,
+phase1_kernel(BuildDev B, int64_t group_size, int64_t g0, int64_t g1,
               const __grid_constant__ CUtensorMap tmap) {
   B.g.tmap = &tmap;
   extern __shared__ __align__(128) uint8_t smem[];
   const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int64_t gi = int64_t(blockIdx.x) * kBuildWarps + w;
-  if (gi >= ngroups) return;
+  const int64_t gi = g0 + int64_t(blockIdx.x) * kBuildWarps + w;   // groups [g0, g1)
+  if (gi >= g1) return;
   WarpSmem ws = carve_warp_smem(
       smem + size_t(w) * warp_smem_bytes(B.l_build, TPL, NV4, B.g.d4, kBuildStageRounds),
       B.l_build, TPL, NV4, B.g.d4, kBuildStageRounds);
@@ -173,18 +175,24 @@ phase1_kernel(BuildDev B, int64_t group_size, int64_t ngroups,
 }
 
 // ------------------------------------------------------------------ K3
-// Phase 2 Step 1 (Alg. 2 lines 10-17) + the counting half of K4.
+// Phase 2 Step 1 (Alg. 2 lines 10-17) + the counting half of K4, for
+// the vertices [v0, v1) of P_i = [lo, hi).  Fused form (F_ids == nullptr, one GPU):
+// v's row, its E slots and the in-degree counts are written here.  Staged form
+// (multi-GPU build): only the new forward row F (first d_min) is written, to
+// F_ids / F_dists [(v - v0)][d_min]; apply_forward_kernel consumes the F of all of
+// P_i after the exchange.
 template <int NV4, int TPL, bool L2>
 __global__ void __launch_bounds__(kBuildWarps * 32)
-round_search_kernel(BuildDev B, int64_t lo, int64_t hi, int32_t* __restrict__ Eu,
+round_search_kernel(BuildDev B, int64_t lo, int64_t v0, int64_t v1, int32_t* __restrict__ Eu,
                     float* __restrict__ Ed, int32_t* __restrict__ indeg,
                     int32_t* __restrict__ touched, int32_t* __restrict__ counters,
+                    int32_t* __restrict__ F_ids, float* __restrict__ F_dists,
                     const __grid_constant__ CUtensorMap tmap, const UpperLayers U, int layer) {
   B.g.tmap = &tmap;
   extern __shared__ __align__(128) uint8_t smem[];
   const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int64_t v = lo + int64_t(blockIdx.x) * kBuildWarps + w;
-  if (v >= hi) return;
+  const int64_t v = v0 + int64_t(blockIdx.x) * kBuildWarps + w;
+  if (v >= v1) return;
   WarpSmem ws = carve_warp_smem(
       smem + size_t(w) * warp_smem_bytes(B.l_build, TPL, NV4, B.g.d4, kBuildStageRounds),
       B.l_build, TPL, NV4, B.g.d4, kBuildStageRounds);
@@ -220,11 +228,20 @@ round_search_kernel(BuildDev B, int64_t lo, int64_t hi, int32_t* __restrict__ Eu
   const int nf = cs + cg < dm ? cs + cg : dm;
   int32_t* row = B.gid + size_t(v) * B.g.d_max;
   float* rowd = B.gdist + size_t(v) * B.g.d_max;
-  for (int j = lane; j < B.g.d_max; j += 32) {   // v's Phase-1 backward edges are dropped (R-C15)
-    if (j >= nf) { row[j] = -1; rowd[j] = __int_as_float(0x7f800000); }
+  const bool staged = F_ids != nullptr;
+  if (staged) {
+    for (int j = lane; j < dm; j += 32)
+      if (j >= nf) {
+        F_ids[size_t(v - v0) * dm + j] = -1;
+        F_dists[size_t(v - v0) * dm + j] = __int_as_float(0x7f800000);
+      }
+  } else {
+    for (int j = lane; j < B.g.d_max; j += 32) {   // v's Phase-1 backward edges are dropped (R-C15)
+      if (j >= nf) { row[j] = -1; rowd[j] = __int_as_float(0x7f800000); }
+    }
+    for (int j = lane; j < dm; j += 32)
+      if (j >= nf) Eu[slot0 + j] = -1;
   }
-  for (int j = lane; j < dm; j += 32)
-    if (j >= nf) Eu[slot0 + j] = -1;
   for (int i = lane; i < cs + cg; i += 32) {
     uint64_t key;
     int rank = 0;
@@ -240,12 +257,47 @@ round_search_kernel(BuildDev B, int64_t lo, int64_t hi, int32_t* __restrict__ Eu
     if (rank < dm) {
       const int32_t u = key_id(key);
       const float dd = key_dist(key);
+      if (staged) {
+        F_ids[size_t(v - v0) * dm + rank] = u;
+        F_dists[size_t(v - v0) * dm + rank] = dd;
+        continue;
+      }
       row[rank] = u;
       rowd[rank] = dd;
       // line 17: E := E u (u -> v, delta(u, v)) in a fixed slot
       Eu[slot0 + rank] = u;
       Ed[slot0 + rank] = dd;
       if (atomicAdd(&indeg[u], 1) == 0) touched[atomicAdd(&counters[0], 1)] = u;
+    }
+  }
+}
+
+// Staged form, after the exchange: the F of every v in P_i = [lo, hi) becomes v's
+// row (R-C15) and its E slots (line 17), and the in-degrees are counted -- exactly
+// what the fused round_search_kernel writes.  One warp per v.
+static __global__ void apply_forward_kernel(const int32_t* __restrict__ F_ids,
+                                            const float* __restrict__ F_dists, int64_t lo,
+                                            int64_t hi, int d_min, int d_max,
+                                            int32_t* __restrict__ gid, float* __restrict__ gdist,
+                                            int32_t* __restrict__ Eu, float* __restrict__ Ed,
+                                            int32_t* __restrict__ indeg,
+                                            int32_t* __restrict__ touched,
+                                            int32_t* __restrict__ counters) {
+  const int lane = threadIdx.x & 31;
+  const int64_t nwarps = int64_t(gridDim.x) * (blockDim.x >> 5);
+  for (int64_t v = lo + int64_t(blockIdx.x) * (blockDim.x >> 5) + (threadIdx.x >> 5); v < hi;
+       v += nwarps) {
+    const size_t f0 = size_t(v - lo) * d_min;
+    for (int j = lane; j < d_max; j += 32) {
+      const int32_t u = j < d_min ? F_ids[f0 + j] : -1;
+      const float dd = j < d_min ? F_dists[f0 + j] : __int_as_float(0x7f800000);
+      gid[size_t(v) * d_max + j] = u;
+      gdist[size_t(v) * d_max + j] = u >= 0 ? dd : __int_as_float(0x7f800000);
+      if (j < d_min) {
+        Eu[f0 + j] = u;
+        Ed[f0 + j] = dd;
+        if (u >= 0 && atomicAdd(&indeg[u], 1) == 0) touched[atomicAdd(&counters[0], 1)] = u;
+      }
     }
   }
 }
@@ -334,13 +386,6 @@ static cudaError_t set_smem_attrs() {
   });
 }
 
-template <typename T>
-struct DevBuf {
-  T* p = nullptr;
-  cudaError_t alloc(size_t count) { return cudaMalloc(&p, std::max<size_t>(count, 1) * sizeof(T)); }
-  ~DevBuf() { if (p) cudaFree(p); }
-};
-
 #define GANNS_TRY(...)                                           \
   do {                                                           \
     cudaError_t _e = (__VA_ARGS__);                              \
@@ -355,117 +400,156 @@ static __global__ void fill_rows_kernel(int32_t* ids, float* dists, int64_t coun
   }
 }
 
+// The state of one Algorithm-2 construction (BuildState, ganns_internal.h) for
+// this (NV4, TPL, L2) instance: the kernels' argument block and launch shapes.
+struct BuildDevState {
+  BuildDev B;
+  UpperLayers U;
+  size_t smem;
+};
+
 template <int NV4, int TPL, bool L2>
-static int build_t(BuildArgs& a, cudaStream_t s) {
+static int phase1_t(BuildState& st, int64_t g0, int64_t g1, cudaStream_t s) {
+  auto* ds = static_cast<BuildDevState*>(st.dev);
+  if (g1 <= g0) return 0;
+  // all local graphs of [g0, g1) in parallel, one warp per group (lines 2-8)
+  phase1_kernel<NV4, TPL, L2><<<unsigned((g1 - g0 + kBuildWarps - 1) / kBuildWarps),
+                                kBuildWarps * 32, ds->smem, s>>>(ds->B, st.S, g0, g1, st.tmap);
+  count_launch();
+  GANNS_TRY(cudaGetLastError());
+  return 0;
+}
+
+template <int NV4, int TPL, bool L2>
+static int round_search_t(BuildState& st, int64_t i, int64_t v0, int64_t v1, int32_t* f_ids,
+                          float* f_dists, cudaStream_t s) {
+  auto* ds = static_cast<BuildDevState*>(st.dev);
+  const int64_t lo = i * st.S;
+  if (v1 <= v0) return 0;
+  if (f_ids == nullptr)   // fused form: counters of this round's GatherScatter start at 0
+    GANNS_TRY(cudaMemsetAsync(st.counters, 0, sizeof(int32_t) * 2, s));
+  round_search_kernel<NV4, TPL, L2><<<unsigned((v1 - v0 + kBuildWarps - 1) / kBuildWarps),
+                                      kBuildWarps * 32, ds->smem, s>>>(
+      ds->B, lo, v0, v1, st.Eu, st.Ed, st.indeg, st.touched, st.counters, f_ids, f_dists, st.tmap,
+      ds->U, st.a.layer);
+  count_launch();
+  GANNS_TRY(cudaGetLastError());
+  return 0;
+}
+
+// Steps 2-3 of round i (lines 19-22) after the E slots and in-degrees are in place.
+template <int TPL>
+static int round_merge_t(BuildState& st, int64_t i, cudaStream_t s) {
+  const int64_t lo = i * st.S, hi = std::min(lo + st.S, st.a.n);
+  const int64_t nslots = (hi - lo) * st.a.d_min;
+  const unsigned gs = unsigned(std::min<int64_t>((nslots + 255) / 256, 148 * 4));
+  alloc_segments_kernel<<<gs, 256, 0, s>>>(st.touched, st.indeg, st.segoff, st.counters);
+  scatter_edges_kernel<<<gs, 256, 0, s>>>(st.Eu, st.Ed, nslots, st.a.d_min, lo, st.segoff,
+                                          st.fill, st.seg);
+  const unsigned gm = unsigned(std::min<int64_t>((nslots + kBuildWarps - 1) / kBuildWarps, 148 * 8));
+  round_merge_kernel<TPL><<<gm, kBuildWarps * 32, 0, s>>>(st.a.out_nbr, st.gdist, st.a.d_max,
+                                                         st.touched, st.indeg, st.fill,
+                                                         st.segoff, st.seg, st.counters);
+  count_launch(3);
+  GANNS_TRY(cudaGetLastError());
+  return 0;
+}
+
+template <int TPL>
+static int round_apply_t(BuildState& st, int64_t i, const int32_t* f_ids, const float* f_dists,
+                         cudaStream_t s) {
+  const int64_t lo = i * st.S, hi = std::min(lo + st.S, st.a.n);
+  GANNS_TRY(cudaMemsetAsync(st.counters, 0, sizeof(int32_t) * 2, s));
+  apply_forward_kernel<<<unsigned(std::min<int64_t>((hi - lo + 7) / 8, 148 * 8)), 256, 0, s>>>(
+      f_ids, f_dists, lo, hi, st.a.d_min, st.a.d_max, st.a.out_nbr, st.gdist, st.Eu, st.Ed,
+      st.indeg, st.touched, st.counters);
+  count_launch();
+  GANNS_TRY(cudaGetLastError());
+  return round_merge_t<TPL>(st, i, s);
+}
+
+template <int NV4, int TPL, bool L2>
+static int begin_t(BuildState& st, cudaStream_t s) {
   GANNS_TRY(set_smem_attrs<NV4, TPL, L2>());
+  BuildArgs& a = st.a;
   const int64_t n = a.n, S = a.group_size;
-  const int64_t ngroups = (n + S - 1) / S;
   const int dm = a.d_min, dmax = a.d_max;
-  DevBuf<float> gdist, gpd, Ed;
-  DevBuf<int32_t> gpid, Eu, indeg, fill, segoff, touched, counters;
-  DevBuf<uint64_t> seg;
-  DevBuf<unsigned long long> stats;
-  GANNS_TRY(gdist.alloc(size_t(n) * dmax));
-  GANNS_TRY(gpid.alloc(size_t(n) * dm));
-  GANNS_TRY(gpd.alloc(size_t(n) * dm));
-  GANNS_TRY(Eu.alloc(size_t(S) * dm));
-  GANNS_TRY(Ed.alloc(size_t(S) * dm));
-  GANNS_TRY(indeg.alloc(size_t(n)));
-  GANNS_TRY(fill.alloc(size_t(n)));
-  GANNS_TRY(segoff.alloc(size_t(n)));
-  GANNS_TRY(touched.alloc(size_t(S) * dm));
-  GANNS_TRY(seg.alloc(size_t(S) * dm));
-  GANNS_TRY(counters.alloc(2));
-  GANNS_TRY(stats.alloc(3));
-  GANNS_TRY(cudaMemsetAsync(indeg.p, 0, sizeof(int32_t) * n, s));
-  GANNS_TRY(cudaMemsetAsync(fill.p, 0, sizeof(int32_t) * n, s));
-  GANNS_TRY(cudaMemsetAsync(stats.p, 0, sizeof(unsigned long long) * 3, s));
-  fill_rows_kernel<<<148 * 8, 256, 0, s>>>(a.out_nbr, gdist.p, n * dmax);
-  fill_rows_kernel<<<148 * 8, 256, 0, s>>>(gpid.p, gpd.p, n * dm);
+  st.S = S;
+  st.ngroups = (n + S - 1) / S;
+  auto* ds = new (std::nothrow) BuildDevState();
+  if (!ds) return fail(GANNS_ENOMEM, "host allocation failed");
+  st.dev = ds;
+  st.dev_free = [](void* p) { delete static_cast<BuildDevState*>(p); };
+  auto alloc = [](auto*& p, size_t count) {
+    return cudaMalloc(&p, std::max<size_t>(count, 1) * sizeof(*p));
+  };
+  GANNS_TRY(alloc(st.gdist, size_t(n) * dmax));
+  GANNS_TRY(alloc(st.gpid, size_t(n) * dm));
+  GANNS_TRY(alloc(st.gpd, size_t(n) * dm));
+  GANNS_TRY(alloc(st.Eu, size_t(S) * dm));
+  GANNS_TRY(alloc(st.Ed, size_t(S) * dm));
+  GANNS_TRY(alloc(st.indeg, size_t(n)));
+  GANNS_TRY(alloc(st.fill, size_t(n)));
+  GANNS_TRY(alloc(st.segoff, size_t(n)));
+  GANNS_TRY(alloc(st.touched, size_t(S) * dm));
+  GANNS_TRY(alloc(st.seg, size_t(S) * dm));
+  GANNS_TRY(alloc(st.counters, 2));
+  GANNS_TRY(alloc(st.stats, 3));
+  GANNS_TRY(cudaMemsetAsync(st.indeg, 0, sizeof(int32_t) * n, s));
+  GANNS_TRY(cudaMemsetAsync(st.fill, 0, sizeof(int32_t) * n, s));
+  GANNS_TRY(cudaMemsetAsync(st.stats, 0, sizeof(unsigned long long) * 3, s));
+  fill_rows_kernel<<<148 * 8, 256, 0, s>>>(a.out_nbr, st.gdist, n * dmax);
+  fill_rows_kernel<<<148 * 8, 256, 0, s>>>(st.gpid, st.gpd, n * dm);
   count_launch(2);
   GANNS_TRY(cudaGetLastError());
 
-  BuildDev B;
+  BuildDev& B = ds->B;
   B.g = GraphView{a.out_nbr, a.X, nullptr, n, dmax, a.d / 4, a.metric};
-  CUtensorMap tmap;
-  GANNS_TRY(uses_tma(NV4) ? encode_row_tmap(a.X, n, a.d, &tmap) : zero_tmap(&tmap));
+  GANNS_TRY(uses_tma(NV4) ? encode_row_tmap(a.X, n, a.d, &st.tmap) : zero_tmap(&st.tmap));
   B.gid = a.out_nbr;
-  B.gdist = gdist.p;
-  B.gpid = gpid.p;
-  B.gpd = gpd.p;
+  B.gdist = st.gdist;
+  B.gpid = st.gpid;
+  B.gpd = st.gpd;
   B.d_min = dm;
   B.l_build = a.l_build;
   B.e_build = a.e_build;
   B.l_local = a.l_local > 0 ? a.l_local : a.l_build;
   B.e_local = a.e_local > 0 ? a.e_local : a.e_build;
-  B.stats = stats.p;
-  const size_t smem =
-      size_t(kBuildWarps) * warp_smem_bytes(a.l_build, TPL, NV4, a.d / 4, kBuildStageRounds);
-  if (smem > 227 * 1024) return fail(-4, "build: shared memory per CTA exceeds 227 KB");
-
-  // Phase 1 (lines 2-8): all local graphs in parallel, one warp per group
-  phase1_kernel<NV4, TPL, L2><<<unsigned((ngroups + kBuildWarps - 1) / kBuildWarps),
-                                kBuildWarps * 32, smem, s>>>(B, S, ngroups, tmap);
-  count_launch();
-  GANNS_TRY(cudaGetLastError());
-
-  // Phase 2 (lines 9-22): merge P_1..P_t into G_0, one round per group
-  UpperLayers U;
-  U.top = a.upper.top;
+  B.stats = st.stats;
+  ds->smem = size_t(kBuildWarps) * warp_smem_bytes(a.l_build, TPL, NV4, a.d / 4, kBuildStageRounds);
+  if (ds->smem > 227 * 1024) return fail(GANNS_ENOTSUP, "build: shared memory per CTA exceeds 227 KB");
+  ds->U.top = a.upper.top;
   for (int j = 0; j < kMaxLayers; ++j) {
-    U.nbr[j] = a.upper.nbr[j];
-    U.n[j] = a.upper.n[j];
+    ds->U.nbr[j] = a.upper.nbr[j];
+    ds->U.n[j] = a.upper.n[j];
   }
-  int64_t rounds = 0;
-  const int64_t last = a.max_rounds < 0 ? ngroups - 1 : std::min<int64_t>(ngroups - 1, a.max_rounds);
-  for (int64_t i = 1; i <= last; ++i) {
-    const int64_t lo = i * S, hi = std::min(lo + S, n);
-    const int64_t nv = hi - lo, nslots = nv * dm;
-    GANNS_TRY(cudaMemsetAsync(counters.p, 0, sizeof(int32_t) * 2, s));
-    round_search_kernel<NV4, TPL, L2><<<unsigned((nv + kBuildWarps - 1) / kBuildWarps),
-                                        kBuildWarps * 32, smem, s>>>(
-        B, lo, hi, Eu.p, Ed.p, indeg.p, touched.p, counters.p, tmap, U, a.layer);
-    const unsigned gs = unsigned(std::min<int64_t>((nslots + 255) / 256, 148 * 4));
-    alloc_segments_kernel<<<gs, 256, 0, s>>>(touched.p, indeg.p, segoff.p, counters.p);
-    scatter_edges_kernel<<<gs, 256, 0, s>>>(Eu.p, Ed.p, nslots, dm, lo, segoff.p, fill.p, seg.p);
-    const unsigned gm = unsigned(std::min<int64_t>((nslots + kBuildWarps - 1) / kBuildWarps, 148 * 8));
-    round_merge_kernel<TPL><<<gm, kBuildWarps * 32, 0, s>>>(a.out_nbr, gdist.p, dmax, touched.p,
-                                                           indeg.p, fill.p, segoff.p, seg.p,
-                                                           counters.p);
-    count_launch(4);
-    GANNS_TRY(cudaGetLastError());
-    ++rounds;
-  }
-  unsigned long long hs[3];
-  GANNS_TRY(cudaMemcpyAsync(hs, stats.p, sizeof(hs), cudaMemcpyDeviceToHost, s));
-  GANNS_TRY(cudaStreamSynchronize(s));
-  a.stats[0] = hs[0];
-  a.stats[1] = hs[1];
-  a.stats[2] = hs[2];
-  a.stats[3] = uint64_t(rounds);
+  st.phase1 = phase1_t<NV4, TPL, L2>;
+  st.round_search = round_search_t<NV4, TPL, L2>;
+  st.round_merge = round_merge_t<TPL>;
+  st.round_apply = round_apply_t<TPL>;
   return 0;
 }
 
 template <int NV4, int TPL>
-static int build_m(BuildArgs& a, cudaStream_t s) {
+static int begin_m(BuildState& st, cudaStream_t s) {
 #ifdef GANNS_DEV_ONE
-  return build_t<NV4, TPL, true>(a, s);
+  return begin_t<NV4, TPL, true>(st, s);
 #endif
-  return a.metric == 0 ? build_t<NV4, TPL, true>(a, s) : build_t<NV4, TPL, false>(a, s);
+  return st.a.metric == 0 ? begin_t<NV4, TPL, true>(st, s) : begin_t<NV4, TPL, false>(st, s);
 }
 template <int NV4>
-int run_build_nv(BuildArgs& a, cudaStream_t s) {
+int build_begin_nv(BuildState& st, cudaStream_t s) {
 #ifdef GANNS_DEV_ONE
-  return build_m<NV4, 1>(a, s);
+  return begin_m<NV4, 1>(st, s);
 #endif
-  switch (tpl_for(a.d_max)) {
-    case 1: return build_m<NV4, 1>(a, s);
-    case 2: return build_m<NV4, 2>(a, s);
-    case 4: return build_m<NV4, 4>(a, s);
+  switch (tpl_for(st.a.d_max)) {
+    case 1: return begin_m<NV4, 1>(st, s);
+    case 2: return begin_m<NV4, 2>(st, s);
+    case 4: return begin_m<NV4, 4>(st, s);
   }
-  return fail(-4, "unsupported degree");
+  return fail(GANNS_ENOTSUP, "unsupported degree");
 }
 
-template int run_build_nv<GANNS_NV4>(BuildArgs&, cudaStream_t);
+template int build_begin_nv<GANNS_NV4>(BuildState&, cudaStream_t);
 
 }  // namespace ganns

@@ -6,6 +6,7 @@
 #include <atomic>
 #include <cstdint>
 #include <string>
+#include <vector>
 
 struct ganns_graph {
   int32_t* nbr = nullptr;   // device [n][d_max]
@@ -138,9 +139,44 @@ struct BuildArgs {
   UpperLayersHost upper;   // HNSW: finished layers above `layer` (top = 0: plain NSW)
   int layer = 0;
 };
-int run_build(BuildArgs& a, cudaStream_t s);
+// One Algorithm-2 construction, step by step (build.cu drives it; the per-instance
+// operations come from build_inst.cu).  Device scratch is owned by the state.
+struct BuildState {
+  BuildArgs a{};
+  int64_t S = 0, ngroups = 0;
+  float* gdist = nullptr;      // [n][d_max] distance half of the build-form rows
+  int32_t* gpid = nullptr;     // G' [n][d_min]
+  float* gpd = nullptr;
+  int32_t* Eu = nullptr;       // E of one round [s][d_min] (fixed slots)
+  float* Ed = nullptr;
+  int32_t* indeg = nullptr;    // GatherScatter counters [n]
+  int32_t* fill = nullptr;
+  int32_t* segoff = nullptr;
+  int32_t* touched = nullptr;  // [s * d_min]
+  uint64_t* seg = nullptr;     // [s * d_min]
+  int32_t* counters = nullptr; // [2]
+  unsigned long long* stats = nullptr;   // [3] iterations, comps, searches
+  CUtensorMap tmap;
+  void* dev = nullptr;                   // instance-private block (build_inst.cu)
+  void (*dev_free)(void*) = nullptr;
+  int device = 0;
+  // operations of the (NV4, TPL, L2) instance
+  int (*phase1)(BuildState&, int64_t g0, int64_t g1, cudaStream_t) = nullptr;
+  int (*round_search)(BuildState&, int64_t i, int64_t v0, int64_t v1, int32_t* f_ids,
+                      float* f_dists, cudaStream_t) = nullptr;
+  int (*round_merge)(BuildState&, int64_t i, cudaStream_t) = nullptr;
+  int (*round_apply)(BuildState&, int64_t i, const int32_t* f_ids, const float* f_dists,
+                     cudaStream_t) = nullptr;
+  // staged-API bookkeeping: groups whose rows are final for Phase 1 (built here or
+  // imported), and the next Phase-2 round
+  std::vector<uint8_t> group_ready;
+  int64_t next_round = 1;
+  ~BuildState();
+};
+int build_begin(BuildState& st, cudaStream_t s);   // scratch + instance operations
 template <int NV4>
-int run_build_nv(BuildArgs& a, cudaStream_t s);
+int build_begin_nv(BuildState& st, cudaStream_t s);
+int run_build(BuildArgs& a, cudaStream_t s);       // the whole construction on one GPU
 
 int run_knn(const float* X, int64_t n, int d, int metric, int K, const int32_t* init_dev,
             int max_iters, int32_t* out_ids, int* iters_out, int64_t* changed_last,

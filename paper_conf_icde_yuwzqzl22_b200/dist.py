@@ -158,6 +158,66 @@ def gpu_replicated_search(graph, points: torch.Tensor, queries: torch.Tensor, k:
                              gather=gather, group=group)
 
 
+def _comm(t: torch.Tensor, group=None) -> torch.Tensor:
+    """gloo collectives run on host tensors (NCCL on device tensors)."""
+    if t.is_cuda and dist.get_backend(group) == "gloo":
+        return t.cpu()
+    return t
+
+
+def _gather_blocks(blocks, counts, group=None):
+    """All-gather per-rank row blocks (tuples of tensors with `counts[r]` rows on rank
+    r) in rank order; every tensor comes back on the device of the local block."""
+    dev = blocks[0].device
+    out = []
+    for t in blocks:
+        out.append(_all_gather_rows(_comm(t, group), counts, group).to(dev))
+    return out
+
+
+def build_distributed(builder, group=None):
+    """Algorithm 2 over the ranks of `group` (NEXT-2; the paper's Remarks,
+    P:299: each working unit builds local graphs and runs its share of a round's
+    searches).  `builder` is one rank's replica of the staged construction
+    (StagedBuild on a GPU; the tests also drive a CPU one):
+
+      Phase 1  rank r builds groups [r*G/W, (r+1)*G/W) (a group touches only its
+               own rows), then the rows (build form + N') are all-gathered so every
+               replica holds every local graph;
+      Phase 2  round i: rank r searches its contiguous share of P_i
+               (query_slice), the new forward rows F [|P_i|, d_min] are all-gathered
+               in vertex order, and every rank applies the same round (rows of P_i,
+               E, GatherScatter, merges) -- one exchange per round.
+
+    The replicas stay bit-identical to a one-GPU build with the same parameters.
+    Returns builder.finish()."""
+    rank, world = _world(group)
+    S, G, d_min, d_max = builder.info()
+    # ---- Phase 1
+    gb = [query_slice(G, r, world) for r in range(world)]
+    builder.phase1(*gb[rank])
+    if world > 1:
+        vb = [builder.group_rows(*gb[r]) for r in range(world)]
+        counts = [b - a for a, b in vb]
+        rows = _gather_blocks(builder.export_rows(*vb[rank]), counts, group)
+        off = 0
+        for r in range(world):
+            if r != rank and counts[r] > 0:
+                builder.import_rows(vb[r][0], vb[r][1],
+                                    tuple(t[off:off + counts[r]].contiguous() for t in rows))
+            off += counts[r]
+    # ---- Phase 2, one exchange per round
+    for i in range(1, G):
+        lo, hi = builder.group_rows(i, i + 1)
+        sl = [query_slice(hi - lo, r, world) for r in range(world)]
+        a, b = sl[rank]
+        f = builder.round_search(i, lo + a, lo + b)
+        if world > 1:
+            f = _gather_blocks(f, [y - x for x, y in sl], group)
+        builder.round_apply(i, *f)
+    return builder.finish()
+
+
 def max_over_ranks(value: float, device=None, group=None) -> float:
     """Max of a per-rank scalar (timings are reported as the max over ranks)."""
     rank, world = _world(group)

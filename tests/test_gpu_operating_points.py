@@ -7,7 +7,7 @@
   of the bench (tolerance).
 * C3: d = 960, the warp-group kernel (search_group_kernel) at l = 320.
 * C2: the full 1M-point build with the bench's parameters (l_build 128,
-  l_local 64, auto group size 1536) bit-exact against the oracle's Algorithm 2
+  l_local 32, auto group size 1536) bit-exact against the oracle's Algorithm 2
   (all host cores; the arithmetic is the sequential one), then the search at
   the bench's operating point (l 128, e 109) on that graph.
 
@@ -117,15 +117,15 @@ def test_c3_group_kernel_l320_fullsize_sampled():
 @pytest.mark.slow
 def test_c2_fullsize_build_bitexact_and_operating_point():
     """BASELINE configs[1]: the bench's build (1M x 128, degree 32, l_build 128,
-    l_local 64, auto group size = 1536, 651 Phase-2 rounds) == the oracle's
+    l_local 32, auto group size = 1536, 651 Phase-2 rounds) == the oracle's
     Algorithm 2, adjacency and build counters; then the bench's operating point
     (l 128, e 109) searched on it in one launch, sampled queries bit-exact."""
     cfg = syn.CONFIGS["C2"]
     X, Q = syn.points(cfg), syn.queries(cfg)
     Xd = cu(X)
-    graph = g.build(Xd, degree=cfg.degree, l_build=128, l_local=64)
+    graph = g.build(Xd, degree=cfg.degree, l_build=128, l_local=32)
     adj = graph.adjacency()
-    ref, _, st = oracle.alg2(X, cfg.degree // 2, cfg.degree, 1536, l_build=128, l_local=64,
+    ref, _, st = oracle.alg2(X, cfg.degree // 2, cfg.degree, 1536, l_build=128, l_local=32,
                              threads=oracle.ncores())
     bad = np.argwhere((adj != ref).any(1)).ravel()
     assert len(bad) == 0, f"{len(bad)} rows differ, first {bad[:5]}"

@@ -16,7 +16,7 @@ ap.add_argument("--config", default="C2")
 ap.add_argument("--n", type=int, default=0)
 ap.add_argument("--group", type=int, default=1536)
 ap.add_argument("--l-build", type=int, default=128)
-ap.add_argument("--l-local", type=int, default=64)
+ap.add_argument("--l-local", type=int, default=32)
 ap.add_argument("--threads", type=int, default=0)
 ap.add_argument("--save", default="")
 a = ap.parse_args()

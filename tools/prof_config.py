@@ -18,7 +18,7 @@ ap.add_argument("--l", type=int, required=True)
 ap.add_argument("--e", type=int, default=0)
 ap.add_argument("--reps", type=int, default=4)
 ap.add_argument("--l-build", type=int, default=128)
-ap.add_argument("--l-local", type=int, default=64)
+ap.add_argument("--l-local", type=int, default=32)
 a = ap.parse_args()
 cfg = syn.CONFIGS[a.config]
 X, Qs = bench.make_workload(cfg, 0, 1)
