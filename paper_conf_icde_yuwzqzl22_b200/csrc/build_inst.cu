@@ -42,6 +42,12 @@
 namespace ganns {
 
 constexpr int kBuildWarps = 1;   // one warp per CTA spreads the latency-bound build searches over all SMs
+#ifndef GANNS_BUILD_PREDICT
+#define GANNS_BUILD_PREDICT 1
+#endif
+// the build searches predict the next exploration and load its adjacency row early
+// (ganns_dev.cuh: warp_search_with, PREDICT)
+constexpr bool kBuildPredict = GANNS_BUILD_PREDICT != 0;
 
 // Insert key kx into a warp-distributed ascending row of d_max keys (TPL per
 // lane, slot j = t*32 + lane); the last key falls off when the row is full
@@ -138,7 +144,7 @@ phase1_kernel(BuildDev B, int64_t group_size, int64_t g0, int64_t g1,
   for (int64_t v = lo + 1; v < hi; ++v) {
     // Step 1 (line 5): v.N, v.N' := Search(G_i, v, d_min), entry = group's first vertex
     SearchStats st;
-    const int cnt = warp_search<NV4, TPL, L2, true>(B.g, B.g.X + size_t(v) * d, int32_t(lo),
+    const int cnt = warp_search<NV4, TPL, L2, true, kBuildPredict>(B.g, B.g.X + size_t(v) * d, int32_t(lo),
                                                     B.l_local, B.e_local, ws, st);
     add_stats(B.stats, st, lane);
     const int m = cnt < B.d_min ? cnt : B.d_min;
@@ -210,7 +216,7 @@ round_search_kernel(BuildDev B, int64_t lo, int64_t v0, int64_t v1, int32_t* __r
     entry = c < lo ? c : 0;
   }
   SearchStats st;
-  const int cnt = warp_search<NV4, TPL, L2, false>(B.g, B.g.X + size_t(v) * d, entry, B.l_build,
+  const int cnt = warp_search<NV4, TPL, L2, false, kBuildPredict>(B.g, B.g.X + size_t(v) * d, entry, B.l_build,
                                                    B.e_build, ws, st);
   add_stats(B.stats, st, lane);
   const int dm = B.d_min;

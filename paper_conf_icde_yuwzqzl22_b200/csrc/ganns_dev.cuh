@@ -174,6 +174,10 @@ constexpr int kWideStageRows = 8;   // d > 256: rows per TMA round (4 rounds per
 #ifndef GANNS_PREFETCH_R2
 #define GANNS_PREFETCH_R2 0
 #endif
+// GANNS_WIDE_HINT: d > 256 -- warm the later TMA rounds' rows in L2 at exploration start
+#ifndef GANNS_WIDE_HINT
+#define GANNS_WIDE_HINT 1
+#endif
 constexpr int kSearchStageRounds = GANNS_SEARCH_ROUNDS;
 constexpr int kBuildStageRounds = 1;
 // wrows: rows per TMA round of the wide (d > 256) form, 1..kWideStageRows (the
@@ -597,9 +601,11 @@ struct WarpDist {
   // soon as the adjacency row is known
   __device__ __forceinline__ void explore_hint(const GraphView& g, int32_t u_mine, int lane,
                                                const WarpSmem& ws) {
+#if GANNS_WIDE_HINT
     if constexpr (!uses_tma(NV4))
       if (u_mine >= 0 && lane >= ws.wrows)
         prefetch_row_l2(g.X + size_t(u_mine) * (g.d4 * 4), uint32_t(g.d4) * 16u);
+#endif
   }
   __device__ __forceinline__ float operator()(const GraphView& g, int32_t u_mine, int lane,
                                               WarpSmem& ws) {
@@ -624,8 +630,12 @@ struct WarpDist {
 // (ascending, explored flags set); returns cnt.  COHERENT: read the graph with
 // coherent loads (the build modifies it inside the same kernel).  DIST computes
 // the bulk distances of one exploration (WarpDist: this warp alone; GroupDist:
-// this warp and its helper warps, search_group.cu).
-template <class DIST, int TPL, bool COHERENT>
+// this warp and its helper warps, search_group.cu).  PREDICT (the latency-bound
+// build searches): right after the lazy check, the vertex explored next is
+// predicted -- the smallest surviving neighbour always enters N, so it is next
+// whenever it precedes the second unexplored entry w -- and its adjacency row is
+// loaded while the sort and merge run.  Results never depend on the prediction.
+template <class DIST, int TPL, bool COHERENT, bool PREDICT = false>
 __device__ int warp_search_with(const GraphView& g, DIST& dist, int32_t entry, int l, int e,
                                 WarpSmem& ws, SearchStats& st) {
   const int lane = threadIdx.x & 31;
@@ -655,11 +665,14 @@ __device__ int warp_search_with(const GraphView& g, DIST& dist, int32_t entry, i
   // row is already in registers (saves one dependent global load per hit)
   int32_t spec_v = -1;
   int32_t spec_u[TPL];
+  int32_t pred_v = -1;      // PREDICT: the vertex predicted after the last lazy check
+  int32_t pred_u[TPL];
   for (;;) {
     // (1) candidate locating: first unexplored entry of N[0..min(e,|N|))
     const int lim = lim_e < cnt ? lim_e : cnt;
     int found = -1;
     int32_t v = 0, w = -1;
+    uint64_t wkey = kKeyInf;   // PREDICT: w's key
     for (int c = hint >> 5; (c << 5) < lim; ++c) {
       int p = (c << 5) + lane;
       uint64_t k = p < lim ? sN[p] : kKeyInf;
@@ -672,6 +685,7 @@ __device__ int warp_search_with(const GraphView& g, DIST& dist, int32_t entry, i
         const unsigned b2 = b & (b - 1);
         const int32_t wk = __shfl_sync(kFull, key_id(k), b2 ? __ffs(b2) - 1 : 0);
         w = b2 ? wk : -1;
+        if constexpr (PREDICT) wkey = b2 ? unflag(shfl64(k, __ffs(b2) - 1)) : kKeyInf;
         break;
       }
     }
@@ -680,18 +694,20 @@ __device__ int warp_search_with(const GraphView& g, DIST& dist, int32_t entry, i
     st.iters++;
     // (2) neighbourhood exploration: T <- out-neighbours of v
     int32_t u[TPL];
-    const bool hit = v == spec_v;
+    const bool hitp = PREDICT && v == pred_v;
+    const bool hit = !hitp && v == spec_v;
     const int32_t* row = g.nbr + size_t(v) * g.d_max;
     const int32_t* wrow = g.nbr + size_t(w < 0 ? 0 : w) * g.d_max;
 #pragma unroll
     for (int t = 0; t < TPL; ++t) {
       const int j = t * 32 + lane;
-      const int32_t ur = (!hit && j < g.d_max) ? load_nbr<COHERENT>(row + j) : -1;
+      const int32_t ur = (!hit && !hitp && j < g.d_max) ? load_nbr<COHERENT>(row + j) : -1;
       const int32_t uw = (w >= 0 && j < g.d_max) ? load_nbr<COHERENT>(wrow + j) : -1;
-      u[t] = hit ? spec_u[t] : ur;
+      u[t] = hitp ? pred_u[t] : hit ? spec_u[t] : ur;
       spec_u[t] = uw;
     }
     spec_v = w;
+    pred_v = -1;
     // (3) bulk distance computation
 #pragma unroll
     for (int t = 0; t < TPL; ++t) dist.explore_hint(g, u[t], lane, ws);
@@ -748,6 +764,25 @@ __device__ int warp_search_with(const GraphView& g, DIST& dist, int32_t entry, i
       hint = found + 1;
       __syncwarp();
       continue;
+    }
+    if constexpr (PREDICT) {
+      uint64_t mk = kKeyInf;
+#pragma unroll
+      for (int t = 0; t < TPL; ++t) mk = cand[t] && key[t] < mk ? key[t] : mk;
+#pragma unroll
+      for (int off = 16; off >= 1; off >>= 1) {
+        const uint64_t o = shfl64(mk, lane ^ off);
+        mk = o < mk ? o : mk;
+      }
+      if (mk < wkey) {   // the smallest survivor precedes w: it is explored next
+        pred_v = key_id(mk);
+        const int32_t* prow = g.nbr + size_t(pred_v) * g.d_max;
+#pragma unroll
+        for (int t = 0; t < TPL; ++t) {
+          const int j = t * 32 + lane;
+          pred_u[t] = j < g.d_max ? load_nbr<COHERENT>(prow + j) : -1;
+        }
+      }
     }
     // (5) sort: rank of each survivor among the survivors, (dist, id) order
     int rT[TPL];
@@ -824,13 +859,13 @@ __device__ int warp_search_with(const GraphView& g, DIST& dist, int32_t entry, i
   return cnt;
 }
 
-template <int NV4, int TPL, bool L2, bool COHERENT>
+template <int NV4, int TPL, bool L2, bool COHERENT, bool PREDICT = false>
 __device__ __forceinline__ int warp_search(const GraphView& g, const float* __restrict__ qrow,
                                            int32_t entry, int l, int e, WarpSmem& ws,
                                            SearchStats& st) {
   WarpDist<NV4, L2> dist;
   dist.load(g, qrow, threadIdx.x & 31);
-  return warp_search_with<WarpDist<NV4, L2>, TPL, COHERENT>(g, dist, entry, l, e, ws, st);
+  return warp_search_with<WarpDist<NV4, L2>, TPL, COHERENT, PREDICT>(g, dist, entry, l, e, ws, st);
 }
 
 // ---------------------------------------------------------------- HNSW
@@ -846,8 +881,16 @@ struct UpperLayers {
 // Greedy descent: the GANNS search with l = e = 1 (the best candidate only) from
 // shuffled id 0 through layers top..stop; returns the vertex reached.  `base`
 // carries the permuted points (and their tensor map) and the degree.
+#ifndef GANNS_DESCEND_NOINLINE
+#define GANNS_DESCEND_NOINLINE 0
+#endif
+#if GANNS_DESCEND_NOINLINE
+#define GANNS_DESCEND_ATTR __noinline__
+#else
+#define GANNS_DESCEND_ATTR
+#endif
 template <int NV4, int TPL, bool L2>
-__device__ int32_t descend(const GraphView& base, const UpperLayers& U, int stop,
+__device__ GANNS_DESCEND_ATTR int32_t descend(const GraphView& base, const UpperLayers& U, int stop,
                            const float* __restrict__ q, WarpSmem& ws,
                            SearchStats* acc = nullptr) {
   int32_t cur = 0;

@@ -155,8 +155,10 @@ struct GroupDist {
   }
   __device__ __forceinline__ void explore_hint(const GraphView& g, int32_t u_mine, int lane,
                                                const WarpSmem& ws) {
+#if GANNS_WIDE_HINT
     if (u_mine >= 0 && lane >= ws.wrows)
       prefetch_row_l2(g.X + size_t(u_mine) * (g.d4 * 4), uint32_t(g.d4) * 16u);
+#endif
   }
   __device__ __forceinline__ float operator()(const GraphView& g, int32_t u_mine, int lane,
                                               WarpSmem& ws) {
