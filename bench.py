@@ -273,10 +273,13 @@ class Pipeline:
     the start of the next one.  Device-timed with CUDA events bracketing all
     streams."""
 
-    def __init__(self, torch, index, Qds, k, nstreams, lo=0, hi=None):
+    def __init__(self, torch, index, Qds, k, nstreams, lo=0, hi=None, replicated=False):
+        """replicated: the steps go through dist.search_replicated (each rank searches
+        its query_slice of the full batch); otherwise the [lo, hi) slice directly."""
         self.torch, self.index, self.k = torch, index, k
         hi = Qds[0].shape[0] if hi is None else hi
-        self.Qds = [q[lo:hi] for q in Qds]          # this rank's slice of every batch
+        self.replicated = replicated
+        self.Qds = Qds if replicated else [q[lo:hi] for q in Qds]   # this rank's slice
         nq = hi - lo
         dev = Qds[0].device
         self.streams = [torch.cuda.Stream(device=dev) for _ in range(max(1, nstreams))]
@@ -310,8 +313,14 @@ class Pipeline:
         def body():
             for i in range(steps):
                 with torch.cuda.stream(self.streams[i % S]):
-                    self.index.search(self.Qds[i % len(self.Qds)], self.k, l, e=e,
-                                      out=self.outs[i % S])
+                    out = self.outs[i % S]
+                    if self.replicated:
+                        from paper_conf_icde_yuwzqzl22_b200 import dist as gdist
+                        gdist.search_replicated(
+                            lambda q: self.index.search(q, self.k, l, e=e, out=out),
+                            self.Qds[i % len(self.Qds)], gather=False)
+                    else:
+                        self.index.search(self.Qds[i % len(self.Qds)], self.k, l, e=e, out=out)
         return self._bracket(body, clk)
 
     def run_host(self, g, Xd, Qhs, steps, l, e):
@@ -582,7 +591,7 @@ def run_ours(args):
     # ---- (l, e) operating point over every query the timed steps search (see
     # select_operating_point); candidates timed as the steps are (pipelined)
     nstreams = streams_for(hi - lo, args.streams) if strong else args.streams
-    pipe = Pipeline(torch, index, Qds, k, nstreams, lo, hi)
+    pipe = Pipeline(torch, index, Qds, k, nstreams, lo, hi, replicated=strong and distributed)
     l_star, e_star, sweep, chosen = select_operating_point(
         torch, index, Qd_all, gt, k, args.target,
         lambda l, e: min(pipe.run(3 * B, l, e) for _ in range(3)))

@@ -11,6 +11,7 @@
 #include <exception>
 #include <mutex>
 #include <new>
+#include <unordered_map>
 #include <vector>
 
 namespace ganns {
@@ -102,26 +103,31 @@ struct HostPipe {
 static std::mutex g_pipe_mu;
 static HostPipe g_pipes[64];
 
-// Ticket counters for the persistent search kernel: a ring of device ints per
-// device, one slot per launch (concurrent launches on different streams get
-// different slots; 4096 launches would have to be in flight to wrap).
+// Ticket counters for the persistent search kernel: one device int per (device,
+// stream).  A launch resets its stream's counter with a memset on that stream, so
+// consecutive launches on one stream are ordered and launches on different
+// streams never share a counter.  Up to kTicketSlots streams per device get
+// their own slot; beyond that, slots are shared round-robin (two launches in
+// flight on two streams that share a slot would race: documented limit).
 constexpr int kTicketSlots = 4096;
 static std::mutex g_ticket_mu;
 static int32_t* g_tickets[64] = {nullptr};
-static std::atomic<uint32_t> g_ticket_next{0};
+static std::unordered_map<cudaStream_t, int32_t> g_ticket_of[64];
 
-int32_t* ticket_slot() {
+int32_t* ticket_slot(cudaStream_t stream) {
   int dev = 0;
   cudaGetDevice(&dev);
   if (dev < 0 || dev >= 64) return nullptr;
-  {
-    std::lock_guard<std::mutex> lock(g_ticket_mu);
-    if (!g_tickets[dev] && cudaMalloc(&g_tickets[dev], sizeof(int32_t) * kTicketSlots) != cudaSuccess) {
-      g_tickets[dev] = nullptr;
-      return nullptr;
-    }
+  std::lock_guard<std::mutex> lock(g_ticket_mu);
+  if (!g_tickets[dev] && cudaMalloc(&g_tickets[dev], sizeof(int32_t) * kTicketSlots) != cudaSuccess) {
+    g_tickets[dev] = nullptr;
+    return nullptr;
   }
-  return g_tickets[dev] + (g_ticket_next.fetch_add(1) % kTicketSlots);
+  auto& m = g_ticket_of[dev];
+  auto it = m.find(stream);
+  if (it == m.end())
+    it = m.emplace(stream, int32_t(m.size() % kTicketSlots)).first;
+  return g_tickets[dev] + it->second;
 }
 
 
@@ -351,7 +357,7 @@ int ganns_search_ex(const ganns_graph* g, const float* points, const float* quer
   if (int rc = validate_search(g, points, queries, nq, k, l, p, out_ids, out_dists, &e, &entry))
     return rc;
   if (nq == 0) return GANNS_OK;
-  int32_t* tk = ticket_slot();
+  int32_t* tk = ticket_slot(static_cast<cudaStream_t>(stream));
   if (!tk) return fail(GANNS_ENOMEM, "ticket allocation failed");
   SearchLaunch a{g->nbr, points, g->n, g->d, g->d_max, g->metric, queries, nq, k, l, e, entry,
                  out_ids, out_dists, p ? p->stats : nullptr, tk};
@@ -422,7 +428,7 @@ int ganns_search_host(const ganns_graph* g, const float* points, const float* qu
     err = cudaMemcpyAsync(P.dq[b], queries_host + size_t(q0) * g->d, sizeof(float) * m * g->d,
                           cudaMemcpyHostToDevice, s);
     if (err != cudaSuccess) break;
-    int32_t* tk = ticket_slot();
+    int32_t* tk = ticket_slot(s);
     if (!tk) return fail(GANNS_ENOMEM, "ticket allocation failed");
     SearchLaunch a{g->nbr, points, g->n, g->d, g->d_max, g->metric, P.dq[b], m, k, l, e, entry,
                    P.dids[b], P.ddst[b], nullptr, tk};
@@ -821,7 +827,7 @@ int ganns_hnsw_search(const ganns_hnsw* h, const float* points, const float* que
       up.nbr[j] = h->upper[j];
       up.n[j] = h->layer_n[j];
     }
-    int32_t* tk = ticket_slot();
+    int32_t* tk = ticket_slot(s);
     if (!tk) return fail(GANNS_ENOMEM, "ticket allocation failed");
     SearchLaunch a{g->nbr, points, g->n, g->d, g->d_max, g->metric, queries, nq, k, l, e, entry,
                    out_ids, out_dists, p ? p->stats : nullptr, tk};
@@ -866,7 +872,7 @@ int ganns_hnsw_search(const ganns_hnsw* h, const float* points, const float* que
     if (entries) cudaFreeAsync(entries, s);
     return cuda_fail(err, "hnsw entries");
   }
-  int32_t* tk = ticket_slot();
+  int32_t* tk = ticket_slot(s);
   if (!tk) return fail(GANNS_ENOMEM, "ticket allocation failed");
   SearchLaunch a{g->nbr, points, g->n, g->d, g->d_max, g->metric, queries, nq, k, l, e, entry,
                  out_ids, out_dists, p ? p->stats : nullptr, tk};

@@ -174,9 +174,13 @@ constexpr int kWideStageRows = 8;   // d > 256: rows per TMA round (4 rounds per
 #ifndef GANNS_PREFETCH_R2
 #define GANNS_PREFETCH_R2 0
 #endif
-// GANNS_WIDE_HINT: d > 256 -- warm the later TMA rounds' rows in L2 at exploration start
+// GANNS_WIDE_HINT: d > 256 -- warm the later TMA rounds' rows in L2 at exploration
+// start.  Off: on C3 (1M x 960) the prefetched rows are evicted before their TMA
+// round reads them (~95 MB of prefetches in flight vs the 126 MB L2) -- with the hint
+// 37.4 GB of DRAM reads per 1K-query step (1.09 x algorithmic) and 189.6K QPS,
+// without it 31.4 GB (0.92 x) and 222.4K QPS (profiles/r02/ab_c3_wide_hint.log)
 #ifndef GANNS_WIDE_HINT
-#define GANNS_WIDE_HINT 1
+#define GANNS_WIDE_HINT 0
 #endif
 constexpr int kSearchStageRounds = GANNS_SEARCH_ROUNDS;
 constexpr int kBuildStageRounds = 1;

@@ -122,7 +122,7 @@ cudaError_t launch_gather_rows(const float* X, const int32_t* perm, int64_t n, i
                                cudaStream_t s);
 cudaError_t launch_relabel(const int32_t* in, const int32_t* perm, int64_t n, int d_max,
                            int32_t* out, cudaStream_t s);
-int32_t* ticket_slot();   // a device int reserved for one launch (ring of slots)
+int32_t* ticket_slot(cudaStream_t stream);   // the search kernel's ticket counter of `stream`
 cudaError_t launch_search(const SearchLaunch& a, cudaStream_t s);
 template <int NV4>
 cudaError_t launch_search_nv(const SearchLaunch& a, cudaStream_t s);

@@ -1,11 +1,12 @@
-// search.cu -- K1, the batched GANNS search kernel (§III-B),
-// plus the multi-GPU helpers K6 (shard top-k merge) and the id offset.
+// search.cu -- dispatch of K1, the batched GANNS search kernel (§III-B,
+// P:193-216; instances in search_inst.cu), the HNSW bookkeeping kernels, and the
+// multi-GPU helpers K6 (shard top-k merge) and the id offset.
 //
-// Launch shape: one warp per query (the paper's block-per-query with n_t = 32,
-// P:201), kWarpsPerBlock queries per CTA, one CTA per kWarpsPerBlock queries;
-// the hardware CTA scheduler back-fills SMs as queries finish.  No global
-// scratch, no atomics: the whole search of a query is one fused warp program
-// (ganns_dev.cuh) and only the top-k leaves the SM.
+// K1's launch shape (search_inst.cu): persistent, grid = SMs x resident CTAs of
+// kSearchWarps warps; every warp takes queries from a per-launch atomic ticket
+// (one warp per query, the paper's n_t = 32) until the batch is
+// exhausted.  No other global scratch: the whole search of a query is one fused
+// warp program (ganns_dev.cuh) and only the top-k leaves the SM.
 #include "ganns_dev.cuh"
 #include "ganns_internal.h"
 

@@ -39,7 +39,7 @@ __global__ void __launch_bounds__(kSearchWarps * 32, NV4 == 1 ? kMinBlocksPerSM 
 search_kernel(GraphView g, const float* __restrict__ Q, int64_t nq, int k, int l, int e,
               int32_t entry, int32_t* __restrict__ out_ids, float* __restrict__ out_dists,
               uint32_t* __restrict__ stats, int32_t* __restrict__ ticket,
-              const int32_t* __restrict__ entries, int wrows,
+              const int32_t* __restrict__ entries, int wrows, int solo,
               const __grid_constant__ CUtensorMap tmap, const __grid_constant__ HnswUpper H,
               const __grid_constant__ CUtensorMap tmap_up) {
   g.tmap = &tmap;
@@ -69,6 +69,18 @@ search_kernel(GraphView g, const float* __restrict__ Q, int64_t nq, int k, int l
     if (lane == 0 && (w & 1) == 0) *ws.pair_flag = 0;
     if (lane == 0) mbar_init(ws.mbar, 1);
     __syncthreads();
+    if (solo && (w & 1)) {
+      // latency mode (a batch that fits one wave at one query per CTA): the odd
+      // warp hands its stage to its partner before taking any query, so every
+      // query runs with one TMA round of 32 rows per exploration -- the same
+      // hand-over as when the ticket runs out (below)
+      fence_proxy_async_smem();
+      __threadfence_block();
+      if (lane == 0) atomicExch(const_cast<int*>(ws.pair_flag), 1);
+      __syncwarp();
+      pair_bar_arrive(ws.pair_bar);
+      return;
+    }
   } else {
     ws = carve_warp_smem(
         smem + size_t(w) * warp_smem_bytes(l, TPL, NV4, g.d4, kSearchStageRounds, wrows), l, TPL,
@@ -151,6 +163,18 @@ static int pick_wide_rows(const SearchLaunch& a, int sms) {
   return kWideStageRows;
 }
 
+// GANNS_SOLO=1 enables the latency mode (off by default: back-to-back small batches
+// on several streams lose their overlap -- each solo batch holds most of the SMs'
+// shared memory; measured 0.61 vs 0.89 per-GPU efficiency on the 8-way strong-scaling
+// proxy, profiles/r02/ab_solo_latency_mode.log)
+static bool solo_enabled() {
+  static const bool on = [] {
+    const char* e = std::getenv("GANNS_SOLO");
+    return e && e[0] == '1';
+  }();
+  return on;
+}
+
 template <int NV4, int TPL, bool L2, bool HNSW = false>
 static cudaError_t launch_t(const SearchLaunch& a, cudaStream_t s) {
   auto kern = search_kernel<NV4, TPL, L2, HNSW>;
@@ -212,12 +236,16 @@ static cudaError_t launch_t(const SearchLaunch& a, cudaStream_t s) {
   if (err != cudaSuccess) return err;
   int64_t blocks = (a.nq + kSearchWarps - 1) / kSearchWarps;
   const int64_t resident = int64_t(sms) * (per_sm > 0 ? per_sm : 1);
+  // latency mode: when one query per CTA fits in one wave, give each query both
+  // stages of its CTA (one TMA round per exploration, shorter per-query latency)
+  const int solo = kPairStages && uses_tma(NV4) && solo_enabled() && a.nq <= resident ? 1 : 0;
+  if (solo) blocks = a.nq;
   if (blocks > resident) blocks = resident;
   err = cudaMemsetAsync(a.ticket, 0, sizeof(int32_t), s);
   if (err != cudaSuccess) return err;
   kern<<<dim3(unsigned(blocks)), kSearchWarps * 32, smem, s>>>(
       g, a.Q, a.nq, a.k, a.l, a.e, a.entry, a.out_ids, a.out_dists, a.stats, a.ticket, a.entries,
-      wrows, tmap, H, tmap_up);
+      wrows, solo, tmap, H, tmap_up);
   count_launch();
   return cudaGetLastError();
 }
