@@ -29,6 +29,25 @@ int cuda_fail(cudaError_t e, const char* what) {
 }
 void count_launch(uint64_t n) { g_launches.fetch_add(n, std::memory_order_relaxed); }
 
+cudaError_t pool_alloc(void** p, size_t bytes, cudaStream_t s) {
+  static std::atomic<uint64_t> raised{0};
+  cudaError_t e = once_per_device(raised, [] {
+    int dev = 0;
+    cudaMemPool_t mp;
+    cudaError_t r = cudaGetDevice(&dev);
+    if (r == cudaSuccess) r = cudaDeviceGetDefaultMemPool(&mp, dev);
+    uint64_t thr = ~uint64_t(0);
+    if (r == cudaSuccess) r = cudaMemPoolSetAttribute(mp, cudaMemPoolAttrReleaseThreshold, &thr);
+    return r;
+  });
+  if (e != cudaSuccess) return e;
+  return cudaMallocAsync(p, bytes, s);
+}
+
+void pool_free(void* p, cudaStream_t s) {
+  if (p) cudaFreeAsync(p, s);
+}
+
 // cuTensorMapEncodeTiled through the runtime's driver entry point (no link-time
 // dependency on libcuda).  Maps are cached per (pointer, n, d).
 typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*,
@@ -655,7 +674,8 @@ int ganns_build_finish(ganns_build_state* s, void* stream, uint64_t* stats, gann
   }
   *out = s->graph;
   s->graph = nullptr;
-  delete s;   // frees the scratch
+  s->st.stream = cs;   // the scratch returns to the pool in stream order
+  delete s;
   return GANNS_OK;
 }
 
@@ -739,14 +759,15 @@ int ganns_build_hnsw(const float* points, int64_t n, int d, int metric, int degr
   int rc = GANNS_OK;
   uint64_t tot[4] = {0, 0, 0, 0};
   auto cleanup = [&](int code) {
-    cudaFree(Xfull);
-    cudaFree(layer0_shuffled);
+    pool_free(Xfull, s);
+    pool_free(layer0_shuffled, s);
     if (code) ganns_hnsw_free(h);
     return code;
   };
   if (cudaMalloc(&h->perm, sizeof(int32_t) * n) != cudaSuccess ||
-      cudaMalloc(&Xfull, sizeof(float) * size_t(n) * d) != cudaSuccess ||
-      cudaMalloc(&layer0_shuffled, sizeof(int32_t) * size_t(n) * degree) != cudaSuccess)
+      pool_alloc(reinterpret_cast<void**>(&Xfull), sizeof(float) * size_t(n) * d, s) != cudaSuccess ||
+      pool_alloc(reinterpret_cast<void**>(&layer0_shuffled), sizeof(int32_t) * size_t(n) * degree,
+                 s) != cudaSuccess)
     return cleanup(fail(GANNS_ENOMEM, "cudaMalloc(hnsw scratch)"));
   cudaError_t e = cudaMemcpy(h->perm, perm.data(), sizeof(int32_t) * n, cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = launch_gather_rows(points, h->perm, n, d, Xfull, s);

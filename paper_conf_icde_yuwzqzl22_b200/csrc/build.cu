@@ -14,24 +14,19 @@ BuildState::~BuildState() {
   int cur = 0;
   cudaGetDevice(&cur);
   cudaSetDevice(device);
-  cudaFree(gdist);
-  cudaFree(gpid);
-  cudaFree(gpd);
-  cudaFree(Eu);
-  cudaFree(Ed);
-  cudaFree(indeg);
-  cudaFree(fill);
-  cudaFree(segoff);
-  cudaFree(touched);
-  cudaFree(seg);
-  cudaFree(counters);
-  cudaFree(stats);
+  for (void* p : {static_cast<void*>(gdist), static_cast<void*>(gpid), static_cast<void*>(gpd),
+                  static_cast<void*>(Eu), static_cast<void*>(Ed), static_cast<void*>(indeg),
+                  static_cast<void*>(fill), static_cast<void*>(segoff),
+                  static_cast<void*>(touched), static_cast<void*>(seg),
+                  static_cast<void*>(counters), static_cast<void*>(stats)})
+    pool_free(p, stream);
   cudaSetDevice(cur);
   if (dev && dev_free) dev_free(dev);
 }
 
 int build_begin(BuildState& st, cudaStream_t s) {
   cudaGetDevice(&st.device);
+  st.stream = s;
   switch (nv4_for(st.a.d)) {
     case 1: return build_begin_nv<1>(st, s);
 #ifndef GANNS_DEV_NV1

@@ -37,16 +37,21 @@
 #include <algorithm>
 #include <cmath>
 #include <new>
+#include <type_traits>
 #include <vector>
 
 namespace ganns {
 
 constexpr int kBuildWarps = 1;   // one warp per CTA spreads the latency-bound build searches over all SMs
 #ifndef GANNS_BUILD_PREDICT
-#define GANNS_BUILD_PREDICT 1
+#define GANNS_BUILD_PREDICT 0
 #endif
-// the build searches predict the next exploration and load its adjacency row early
-// (ganns_dev.cuh: warp_search_with, PREDICT)
+// GANNS_BUILD_PREDICT=1: the build searches predict the next exploration and load its
+// adjacency row early (ganns_dev.cuh: warp_search_with, PREDICT).  Off: measured on
+// the GPU clock (C2, 8 builds each) Phase 1 0.1244 vs 0.1199 s, Phase 2 0.4256 vs
+// 0.4078 s with / without (profiles/r02/build_phases_predict_ab.log) -- the extra
+// warp-min and load sit on the chain and the hidden adjacency latency is small (the
+// adjacency rows mostly hit L2)
 constexpr bool kBuildPredict = GANNS_BUILD_PREDICT != 0;
 
 // Insert key kx into a warp-distributed ascending row of d_max keys (TPL per
@@ -486,8 +491,11 @@ static int begin_t(BuildState& st, cudaStream_t s) {
   if (!ds) return fail(GANNS_ENOMEM, "host allocation failed");
   st.dev = ds;
   st.dev_free = [](void* p) { delete static_cast<BuildDevState*>(p); };
-  auto alloc = [](auto*& p, size_t count) {
-    return cudaMalloc(&p, std::max<size_t>(count, 1) * sizeof(*p));
+  auto alloc = [s](auto*& p, size_t count) {
+    void* q = nullptr;
+    cudaError_t e = pool_alloc(&q, std::max<size_t>(count, 1) * sizeof(*p), s);
+    p = static_cast<std::remove_reference_t<decltype(p)>>(q);
+    return e;
   };
   GANNS_TRY(alloc(st.gdist, size_t(n) * dmax));
   GANNS_TRY(alloc(st.gpid, size_t(n) * dm));

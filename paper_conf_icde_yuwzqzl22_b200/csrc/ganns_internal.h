@@ -60,6 +60,13 @@ inline cudaError_t once_per_device(std::atomic<uint64_t>& done, F&& set) {
   return e;
 }
 
+// Stream-ordered scratch from the device's default memory pool.  The pool's release
+// threshold is raised once per device, so freed blocks stay mapped for the next
+// build: a cudaMalloc/cudaFree of the build scratch cost 2 ms typically and up to
+// 1 s of host time (profiles/r02/build_phases_host_gap.log), the pool 0.02 ms.
+cudaError_t pool_alloc(void** p, size_t bytes, cudaStream_t s);
+void pool_free(void* p, cudaStream_t s);
+
 void set_error(const std::string& msg);
 int fail(int status, const std::string& msg);
 int cuda_fail(cudaError_t e, const char* what);
@@ -157,6 +164,7 @@ struct BuildState {
   int32_t* counters = nullptr; // [2]
   unsigned long long* stats = nullptr;   // [3] iterations, comps, searches
   CUtensorMap tmap;
+  cudaStream_t stream = nullptr;         // the scratch is stream-ordered on this stream
   void* dev = nullptr;                   // instance-private block (build_inst.cu)
   void (*dev_free)(void*) = nullptr;
   int device = 0;

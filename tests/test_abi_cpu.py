@@ -64,3 +64,27 @@ def test_binding_refuses_mis_shaped_output_buffers():
             g._check_buf(bad, (4, 10), torch.int32, False, "x")
     with pytest.raises(TypeError):   # host tensor where a CUDA one is required
         g._check_buf(ok, (4, 10), torch.int32, True, "x")
+
+
+def test_graph_load_rejects_corrupt_headers_before_allocating(tmp_path):
+    """ganns_graph_load validates the header (n, d, d_max, metric) and the exact file
+    length before any allocation: a hostile n fails with GANNS_EIO (-5), no throw."""
+    import struct
+    lib = ctypes.CDLL(LIB)
+    lib.ganns_graph_load.argtypes = [ctypes.c_char_p, ctypes.c_int, ctypes.POINTER(ctypes.c_void_p)]
+    lib.ganns_graph_load.restype = ctypes.c_int
+    lib.ganns_last_error.restype = ctypes.c_char_p
+    cases = {
+        "huge_n": struct.pack("<8sq4i", b"GANNSG01", 1 << 40, 128, 32, 0, 0),
+        "neg_n": struct.pack("<8sq4i", b"GANNSG01", -5, 128, 32, 0, 0),
+        "bad_d": struct.pack("<8sq4i", b"GANNSG01", 100, 130, 32, 0, 0),
+        "bad_metric": struct.pack("<8sq4i", b"GANNSG01", 100, 128, 32, 7, 0),
+        "truncated": struct.pack("<8sq4i", b"GANNSG01", 100, 128, 32, 0, 0) + b"\0" * 400,
+        "bad_magic": struct.pack("<8sq4i", b"NOTAGRPH", 100, 128, 32, 0, 0),
+    }
+    for name, blob in cases.items():
+        p = tmp_path / f"{name}.bin"
+        p.write_bytes(blob)
+        h = ctypes.c_void_p()
+        assert lib.ganns_graph_load(str(p).encode(), 0, ctypes.byref(h)) == -5, name
+        assert h.value is None

@@ -55,6 +55,8 @@ for r in range(reps):
     t0 = time.perf_counter()
     b = g.StagedBuild(X, degree=32, l_build=128, l_local=32)
     S, G, dm, dx = b.info()
+    torch.cuda.synchronize()
+    tb = time.perf_counter()
     e0 = ev()
     b.phase1(0, G)
     e1 = ev()
@@ -62,11 +64,19 @@ for r in range(reps):
         lo, hi = b.group_rows(i, i + 1)
         b.round_apply(i, *b.round_search(i, lo, hi))
     e2 = ev()
+    e2.synchronize()
+    tf = time.perf_counter()
     gr = b.finish()
     torch.cuda.synchronize()
     t1 = time.perf_counter()
+    t2 = time.perf_counter()
+    del gr
+    torch.cuda.synchronize()
+    t3 = time.perf_counter()
     win = [s for s in samples if t0 <= s[0] <= t1]
-    print(json.dumps({"rep": r, "wall_s": round(t1 - t0, 4),
+    print(json.dumps({"rep": r, "wall_s": round(t1 - t0, 4), "begin_s": round(tb - t0, 4),
+                      "enqueue_to_done_s": round(tf - tb, 4), "finish_s": round(t1 - tf, 4),
+                      "graph_free_s": round(t3 - t2, 4),
                       "phase1_s": round(e0.elapsed_time(e1) / 1e3, 4),
                       "phase2_s": round(e1.elapsed_time(e2) / 1e3, 4),
                       "sm_mhz": statistics.median([s[1] for s in win]) if win else None,
