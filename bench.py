@@ -869,8 +869,10 @@ def run_sharded(args):
     rec = recall_at(ids[:nsub], gt)
     qps = len(Q) * args.steps / t_total
     # DRAM bytes of the same steps (hardware counters, untimed second pass; a
-    # collective inside a profiled range is fine -- it is one pass, no replay)
-    dram = measure_dram(lambda: steps_run(args.steps)[0], local)
+    # collective inside a profiled range is fine -- it is one pass, no replay).  Two
+    # steps (16 shard launches): the profiler's stop failed on a 10-step range (0.55 s)
+    dsteps = min(2, args.steps)
+    dram = measure_dram(lambda: steps_run(dsteps)[0], local)
     # roofline of K1 on the shards (untimed stats pass: the kernel's own counters)
     # per shard launch: the timed region over the launches (they overlap pairwise)
     search_s = t_total / args.steps / max(1, len(shards))
@@ -923,7 +925,7 @@ def run_sharded(args):
         "gpu_launches": int(launches), "clocks": clk.summary(),
         "e2e": {"value": round(e2e_qps, 1), "unit": "queries/s",
                 "h2d_bytes_per_step": int(Q.nbytes), "d2h_bytes_per_step": int(len(Q) * k * 8)},
-        "roofline": roofline(alg_per_launch, search_s, dram, args.steps * max(1, len(shards)), peak,
+        "roofline": roofline(alg_per_launch, search_s, dram, dsteps * max(1, len(shards)), peak,
                              peak_kind,
                              f"ganns::search_kernel on one {per}-row shard (d={cfg.d}, "
                              f"d_max={cfg.degree}, {cfg.metric}); mean over the shard launches",

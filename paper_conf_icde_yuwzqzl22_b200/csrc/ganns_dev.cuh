@@ -742,25 +742,37 @@ __device__ int warp_search_with(const GraphView& g, DIST& dist, int32_t entry, i
     int rN[TPL];
     unsigned cb[TPL];
     int ncand = 0;
+    // the distance halves of N's keys (word 2i + 1 of key i): the lower_bound
+    // compares 32-bit distances only -- one load and one compare per probe, no
+    // flag masking; equal distances (rare) are resolved on the full key after
+    const uint32_t* sNd = reinterpret_cast<const uint32_t*>(sN) + 1;
 #pragma unroll
     for (int t = 0; t < TPL; ++t) {
       cand[t] = u[t] >= 0 && key[t] < worst;
-      // 4-ary lower_bound of key[t] in N[0..cnt): three independent probes per
-      // step; the trip count depends only on cnt (warp-uniform)
+      // 4-ary lower_bound of key[t]'s distance in N[0..cnt): three independent
+      // probes per step; the trip count depends only on cnt (warp-uniform)
       const uint64_t kt = key[t];
+      const uint32_t kd = uint32_t(kt >> 32);
       int base = 0, len = cnt;   // invariant: lower_bound in [base, base + len]
       while (len > 3) {
         const int q = len >> 2;
-        const int c = (unflag(sN[base + q]) < kt ? 1 : 0) + (unflag(sN[base + 2 * q]) < kt ? 1 : 0) +
-                      (unflag(sN[base + 3 * q]) < kt ? 1 : 0);
+        const int c = (sNd[2 * (base + q)] < kd ? 1 : 0) + (sNd[2 * (base + 2 * q)] < kd ? 1 : 0) +
+                      (sNd[2 * (base + 3 * q)] < kd ? 1 : 0);
         base += c * q;
         len = c < 3 ? q : len - 3 * q;
       }
       int r = base;
 #pragma unroll
-      for (int i = 0; i < 3; ++i) r += (i < len && unflag(sN[base + i]) < kt) ? 1 : 0;
+      for (int i = 0; i < 3; ++i) r += (i < len && sNd[2 * (base + i)] < kd) ? 1 : 0;
+      // r = first entry with distance >= kd; entries of equal distance follow in id
+      // order: skip the smaller ids -- then N[r] is the full-key lower_bound
+      uint64_t nk = r < cnt ? unflag(sN[r]) : kKeyInf;
+      while (nk < kt) {
+        ++r;
+        nk = r < cnt ? unflag(sN[r]) : kKeyInf;
+      }
       rN[t] = r;
-      if (r < cnt && unflag(sN[r]) == kt) cand[t] = false;   // lazy check: in N (R-C1)
+      if (nk == kt) cand[t] = false;   // lazy check: in N (R-C1)
       cb[t] = __ballot_sync(kFull, cand[t]);
       ncand += __popc(cb[t]);
     }
@@ -821,33 +833,48 @@ __device__ int warp_search_with(const GraphView& g, DIST& dist, int32_t entry, i
         asm volatile("prefetch.global.L2 [%0];" ::"l"(g.nbr + size_t(u[t]) * g.d_max));
         sT[rT[t]] = key[t];
         atomicOr(&sBM[pos >> 5], 1u << (pos & 31));
-        pmin = pos < pmin ? pos : pmin;
       }
       nins += __popc(__ballot_sync(kFull, ins));
-    }
-#pragma unroll
-    for (int off = 16; off >= 1; off >>= 1) {
-      int o = __shfl_xor_sync(kFull, pmin, off);
-      pmin = o < pmin ? o : pmin;
+      // the smallest survivor (rank 0 among the survivors) always enters N and
+      // has the smallest position of all insertions: pmin = its rank in N
+      const unsigned m0 = __ballot_sync(kFull, cand[t] && rT[t] == 0);
+      if (m0) pmin = __shfl_sync(kFull, rN[t], __ffs(m0) - 1);
     }
     const int ncnt = cnt + ncand < l ? cnt + ncand : l;
     if (nins > 0) {
       __syncwarp();
       st.merged += nins;
       // rebuild N in place from the last chunk down: output p takes the compacted
-      // T entry #(T positions < p) or N[p - #(T positions < p)]
+      // T entry #(T positions < p) or N[p - #(T positions < p)].  Four chunks per
+      // step: every source of a chunk lies at or below it, so reading the four
+      // chunks' sources before writing any of them is safe
       int suffix = 0;   // T positions at or above the current chunk
-      for (int c = (ncnt - 1) >> 5; c >= (pmin >> 5); --c) {
-        const uint32_t word = sBM[c];
-        suffix += __popc(word);
-        const int p = (c << 5) + lane;
-        const bool isT = (word >> lane) & 1u;
-        const int tb = nins - suffix + __popc(word & lanemask_lt());
-        uint64_t val = 0;
-        if (p < ncnt) val = isT ? sT[tb] : sN[p - tb];
+      const int c_lo = pmin >> 5;
+      for (int c0 = (ncnt - 1) >> 5; c0 >= c_lo; c0 -= 4) {
+        uint64_t val[4];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+          const int c = c0 - j;
+          val[j] = 0;
+          if (c >= c_lo) {
+            const uint32_t word = sBM[c];
+            suffix += __popc(word);
+            const int p = (c << 5) + lane;
+            const bool isT = (word >> lane) & 1u;
+            const int tb = nins - suffix + __popc(word & lanemask_lt());
+            if (p < ncnt) val[j] = isT ? sT[tb] : sN[p - tb];
+          }
+        }
         __syncwarp();
-        if (p < ncnt) sN[p] = val;
-        if (lane == 0) sBM[c] = 0u;
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+          const int c = c0 - j;
+          if (c >= c_lo) {
+            const int p = (c << 5) + lane;
+            if (p < ncnt) sN[p] = val[j];
+            if (lane == 0) sBM[c] = 0u;
+          }
+        }
         __syncwarp();
       }
 #if GANNS_LATE_FENCE

@@ -18,7 +18,8 @@ case "$1" in
     echo "bench $cfg rc=$?"; tail -c 600 "gpurun_out/bench_${cfg}.log" ;;
   ncu)
     cfg=$2; l=$3; e=$4
-    timeout 1500 ncu --set full --import-source on --clock-control none -k regex:search -s 2 -c 1 \
+    timeout 1500 ncu --set full --import-source on --clock-control none \
+      -k "regex:^search(_group)?_kernel" -s 2 -c 1 \
       -o "gpurun_out/ncu_${cfg}_l${l}" -f python tools/prof_config.py --config "$cfg" --l "$l" --e "$e" \
       > "gpurun_out/ncu_${cfg}.log" 2>&1
     echo "ncu rc=$?"; tail -3 "gpurun_out/ncu_${cfg}.log" ;;
