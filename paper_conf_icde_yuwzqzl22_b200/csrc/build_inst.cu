@@ -342,16 +342,20 @@ static __global__ void scatter_edges_kernel(const int32_t* __restrict__ Eu, cons
 // ------------------------------------------------------------------ K5
 // Phase 2 Step 3 (Alg. 2 lines 20-22): per distinct u, keep the first
 // d_max of merge(u.N, E segment of u).  Resets the per-u counters for the next round.
+// One warp per u, kMergeWarps per CTA, enough warps for one u each: a warp's work is
+// a dependent chain (row load -> inserts -> store), so fewer warps looping over
+// several u's made K5 latency-bound (28 us per round at 1184 warps).
+constexpr int kMergeWarps = 8;
 template <int TPL>
-__global__ void __launch_bounds__(kBuildWarps * 32)
+__global__ void __launch_bounds__(kMergeWarps * 32)
 round_merge_kernel(int32_t* __restrict__ gid, float* __restrict__ gdist, int d_max,
                    const int32_t* __restrict__ touched, int32_t* __restrict__ indeg,
                    int32_t* __restrict__ fill, const int32_t* __restrict__ segoff,
                    const uint64_t* __restrict__ seg, const int32_t* __restrict__ counters) {
   const int lane = threadIdx.x & 31;
   const int32_t nt = counters[0];
-  const int32_t nwarps = gridDim.x * kBuildWarps;
-  for (int32_t i = blockIdx.x * kBuildWarps + (threadIdx.x >> 5); i < nt; i += nwarps) {
+  const int32_t nwarps = gridDim.x * kMergeWarps;
+  for (int32_t i = blockIdx.x * kMergeWarps + (threadIdx.x >> 5); i < nt; i += nwarps) {
     const int32_t u = touched[i];
     const int32_t m = indeg[u], off = segoff[u];
     uint64_t key[TPL];
@@ -457,8 +461,8 @@ static int round_merge_t(BuildState& st, int64_t i, cudaStream_t s) {
   alloc_segments_kernel<<<gs, 256, 0, s>>>(st.touched, st.indeg, st.segoff, st.counters);
   scatter_edges_kernel<<<gs, 256, 0, s>>>(st.Eu, st.Ed, nslots, st.a.d_min, lo, st.segoff,
                                           st.fill, st.seg);
-  const unsigned gm = unsigned(std::min<int64_t>((nslots + kBuildWarps - 1) / kBuildWarps, 148 * 8));
-  round_merge_kernel<TPL><<<gm, kBuildWarps * 32, 0, s>>>(st.a.out_nbr, st.gdist, st.a.d_max,
+  const unsigned gm = unsigned(std::min<int64_t>((nslots + kMergeWarps - 1) / kMergeWarps, 148 * 16));
+  round_merge_kernel<TPL><<<gm, kMergeWarps * 32, 0, s>>>(st.a.out_nbr, st.gdist, st.a.d_max,
                                                          st.touched, st.indeg, st.fill,
                                                          st.segoff, st.seg, st.counters);
   count_launch(3);
