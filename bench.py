@@ -13,8 +13,10 @@ drain tail of one batch overlaps the start of the next.  They rotate over
 --batches distinct query batches (no step re-reads its predecessor's queries'
 rows from L2); the working set (vectors + graph) is larger than the 126 MB L2, so
 L2 is not flushed.  Inputs are resident in HBM when the timed region starts.
-Under torchrun each rank builds the same deterministic graph and searches its own
-batches (weak scaling, no data-path collective); time = max over ranks.
+Under torchrun each rank builds the same deterministic graph; by default
+each step's fixed 10K-query batch is split over the ranks (strong scaling through
+dist.search_replicated, no data-path collective); --scaling weak gives every rank its
+own batches.  Time = max over ranks.
 
 --impl reference times the CPU oracle (oracle/, plain C, all host cores) on a
 bounded sample of the same queries, same graph, same l.
@@ -63,9 +65,10 @@ def parse():
                     help="CUDA streams the steps alternate over (1 = serialised launches)")
     ap.add_argument("--shard-rows", type=int, default=0,
                     help="C5 only: rows per shard (default: n / shards = 12.5M)")
-    ap.add_argument("--scaling", default="weak", choices=["weak", "strong"],
-                    help="weak: every rank searches its own batches; strong: each step's "
-                         "batch is split over the ranks (dist.query_slice)")
+    ap.add_argument("--scaling", default="strong", choices=["weak", "strong"],
+                    help="strong (default, SURVEY 8(e)): each step's fixed 10K batch is split "
+                         "over the ranks (dist.search_replicated / query_slice); weak: every "
+                         "rank searches its own batches")
     ap.add_argument("--proxy-worlds", default="2,4,8",
                     help="N=1 only: strong-scaling proxy -- time each of the W slices of the "
                          "fixed batch alone on this GPU (max over slices), per W")
