@@ -321,6 +321,16 @@ GANNS_API const char *ganns_last_error(void);
  * process so far (bench evidence for "gpu_launches"). */
 GANNS_API uint64_t ganns_kernel_launches(void);
 
+/* ganns_profile_read -- per-phase cycle counters of the search loop (the
+ * analogue of the paper's time breakdowns, Fig. 7 / Fig. 10), summed
+ * over every search (batched search and build) on the current device since the last
+ * reset: out[0..5] = cycles in candidate locating, neighbourhood exploration,
+ * bulk distance, lazy check, sort, merge (lane 0's clock64 at the phase
+ * boundaries), out[6] = iterations, out[7] = searches.  Syncs the device; reset != 0
+ * zeroes the counters.  GANNS_ENOTSUP unless the library was built with
+ * -DGANNS_PROFILE=1 (tools/build_variants.sh prof -DGANNS_PROFILE=1). */
+GANNS_API int ganns_profile_read(uint64_t *out, int reset);
+
 #ifdef __cplusplus
 }
 #endif

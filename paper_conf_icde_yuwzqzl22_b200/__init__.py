@@ -91,6 +91,8 @@ def _load():
     lib.ganns_last_error.restype = ct.c_char_p
     lib.ganns_kernel_launches.argtypes = []
     lib.ganns_kernel_launches.restype = ct.c_uint64
+    lib.ganns_profile_read.argtypes = [P, i32]
+    lib.ganns_profile_read.restype = ct.c_int
     return lib
 
 
@@ -106,7 +108,8 @@ ABI_SYMBOLS = ("ganns_build", "ganns_search", "ganns_search_ex", "ganns_search_h
                "ganns_hnsw_info", "ganns_hnsw_layer", "ganns_hnsw_perm", "ganns_hnsw_base",
                "ganns_hnsw_free", "ganns_build_knn", "ganns_build_begin", "ganns_build_info",
                "ganns_build_phase1", "ganns_build_rows", "ganns_build_round_search",
-               "ganns_build_round_apply", "ganns_build_finish", "ganns_build_abort")
+               "ganns_build_round_apply", "ganns_build_finish", "ganns_build_abort",
+               "ganns_profile_read")
 
 
 def lib():
@@ -165,6 +168,19 @@ def _check_index_inputs(graph, points: torch.Tensor, queries: torch.Tensor):
 def kernel_launches() -> int:
     """Kernels launched by libganns.so in this process."""
     return int(_lib.ganns_kernel_launches())
+
+
+PROFILE_PHASES = ("locate", "explore", "distance", "lazy_check", "sort", "merge")
+
+
+def profile_read(reset: bool = True):
+    """Per-phase cycle counters of a GANNS_PROFILE library build (ganns_profile_read):
+    dict(phase -> cycles, iterations, searches).  Raises on a normal build."""
+    out = (ct.c_uint64 * 8)()
+    _check(_lib.ganns_profile_read(ct.cast(out, ct.c_void_p), int(reset)))
+    d = {k: int(out[i]) for i, k in enumerate(PROFILE_PHASES)}
+    d["iterations"], d["searches"] = int(out[6]), int(out[7])
+    return d
 
 
 class Graph:

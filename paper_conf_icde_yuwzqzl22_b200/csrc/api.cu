@@ -44,6 +44,23 @@ cudaError_t pool_alloc(void** p, size_t bytes, cudaStream_t s) {
   return cudaMallocAsync(p, bytes, s);
 }
 
+unsigned long long* prof_buffer() {
+#if GANNS_PROFILE
+  static std::mutex mu;
+  static unsigned long long* buf[64] = {nullptr};
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return nullptr;
+  std::lock_guard<std::mutex> lock(mu);
+  if (!buf[dev]) {
+    if (cudaMalloc(&buf[dev], 8 * sizeof(unsigned long long)) != cudaSuccess) return nullptr;
+    cudaMemset(buf[dev], 0, 8 * sizeof(unsigned long long));
+  }
+  return buf[dev];
+#else
+  return nullptr;
+#endif
+}
+
 void pool_free(void* p, cudaStream_t s) {
   if (p) cudaFreeAsync(p, s);
 }
@@ -192,6 +209,16 @@ extern "C" {
 
 const char* ganns_last_error(void) { return g_last_error.c_str(); }
 uint64_t ganns_kernel_launches(void) { return g_launches.load(); }
+
+int ganns_profile_read(uint64_t* out, int reset) {
+  unsigned long long* p = prof_buffer();
+  if (!p) return fail(GANNS_ENOTSUP, "library built without GANNS_PROFILE");
+  if (!out) return fail(GANNS_EINVAL, "out is NULL");
+  cudaError_t e = cudaDeviceSynchronize();
+  if (e == cudaSuccess) e = cudaMemcpy(out, p, 8 * sizeof(uint64_t), cudaMemcpyDeviceToHost);
+  if (e == cudaSuccess && reset) e = cudaMemset(p, 0, 8 * sizeof(uint64_t));
+  return e == cudaSuccess ? GANNS_OK : cuda_fail(e, "ganns_profile_read");
+}
 
 int ganns_graph_info(const ganns_graph* g, int64_t* n, int* d, int* d_max, int* metric) {
   if (int rc = check_graph(g)) return rc;

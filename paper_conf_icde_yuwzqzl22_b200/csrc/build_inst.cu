@@ -523,6 +523,7 @@ static int begin_t(BuildState& st, cudaStream_t s) {
 
   BuildDev& B = ds->B;
   B.g = GraphView{a.out_nbr, a.X, nullptr, n, dmax, a.d / 4, a.metric};
+  B.g.prof = prof_buffer();
   GANNS_TRY(uses_tma(NV4) ? encode_row_tmap(a.X, n, a.d, &st.tmap) : zero_tmap(&st.tmap));
   B.gid = a.out_nbr;
   B.gdist = st.gdist;

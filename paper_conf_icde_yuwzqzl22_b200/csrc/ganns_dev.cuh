@@ -139,7 +139,20 @@ struct GraphView {
   int d_max;
   int d4;               // d / 4
   int metric;           // 0 L2, 1 IP, 2 COSINE
+  // GANNS_PROFILE builds: per-phase cycle counters (ganns_profile_read), else null
+  unsigned long long* prof = nullptr;
 };
+
+// Per-phase timers of the search loop (the analogue of the paper's time
+// breakdowns, Fig. 7, Fig. 10).  Compiled in only with -DGANNS_PROFILE=1
+// (a separate library build): lane 0 of each warp reads clock64() at the phase
+// boundaries and adds the cycles to prof[0..5] = candidate locating, neighbourhood
+// exploration (adjacency row), bulk distance (gather + math), lazy check, sort,
+// merge; prof[6] = iterations, prof[7] = searches.
+#ifndef GANNS_PROFILE
+#define GANNS_PROFILE 0
+#endif
+enum { kProfLocate = 0, kProfExplore, kProfDistance, kProfLazy, kProfSort, kProfMerge };
 
 // Per-search counters (kept in registers, identical to the oracle's stats[0,1,3]).
 struct SearchStats {
@@ -671,6 +684,18 @@ __device__ int warp_search_with(const GraphView& g, DIST& dist, int32_t entry, i
   int32_t spec_u[TPL];
   int32_t pred_v = -1;      // PREDICT: the vertex predicted after the last lazy check
   int32_t pred_u[TPL];
+#if GANNS_PROFILE
+  unsigned long long pc[6] = {0, 0, 0, 0, 0, 0};
+  long long tp = clock64();
+#define GANNS_PROF_MARK(i)          \
+  {                                 \
+    const long long t_ = clock64(); \
+    pc[i] += t_ - tp;               \
+    tp = t_;                        \
+  }
+#else
+#define GANNS_PROF_MARK(i)
+#endif
   for (;;) {
     // (1) candidate locating: first unexplored entry of N[0..min(e,|N|))
     const int lim = lim_e < cnt ? lim_e : cnt;
@@ -696,6 +721,7 @@ __device__ int warp_search_with(const GraphView& g, DIST& dist, int32_t entry, i
     if (found < 0) break;
     __syncwarp();   // the explored mark (one lane's store) is visible to the whole warp
     st.iters++;
+    GANNS_PROF_MARK(kProfLocate);
     // (2) neighbourhood exploration: T <- out-neighbours of v
     int32_t u[TPL];
     const bool hitp = PREDICT && v == pred_v;
@@ -712,6 +738,10 @@ __device__ int warp_search_with(const GraphView& g, DIST& dist, int32_t entry, i
     }
     spec_v = w;
     pred_v = -1;
+#if GANNS_PROFILE
+    if (__ballot_sync(kFull, u[0] >= 0) == 0xdeadbeefu) st.merged += 0;   // waits for the row
+    GANNS_PROF_MARK(kProfExplore);
+#endif
     // (3) bulk distance computation
 #pragma unroll
     for (int t = 0; t < TPL; ++t) dist.explore_hint(g, u[t], lane, ws);
@@ -723,6 +753,7 @@ __device__ int warp_search_with(const GraphView& g, DIST& dist, int32_t entry, i
       st.comps += __popc(__ballot_sync(kFull, u[t] >= 0));
     }
     __syncwarp();   // every lane's stage reads precede the merge's writes of T (it shares the stage)
+    GANNS_PROF_MARK(kProfDistance);
     // (4) lazy check (R-C1): drop entries already in N; entries that
     // cannot enter N (>= its l-th key while N is full) are dropped as well.
     const uint64_t worst = cnt == l ? unflag(sN[l - 1]) : kKeyInf;
@@ -734,6 +765,7 @@ __device__ int warp_search_with(const GraphView& g, DIST& dist, int32_t entry, i
       if (below == 0) {
         hint = found + 1;
         __syncwarp();
+        GANNS_PROF_MARK(kProfLazy);
         continue;
       }
     }
@@ -779,8 +811,10 @@ __device__ int warp_search_with(const GraphView& g, DIST& dist, int32_t entry, i
     if (ncand == 0) {
       hint = found + 1;
       __syncwarp();
+      GANNS_PROF_MARK(kProfLazy);
       continue;
     }
+    GANNS_PROF_MARK(kProfLazy);
     if constexpr (PREDICT) {
       uint64_t mk = kKeyInf;
 #pragma unroll
@@ -822,6 +856,7 @@ __device__ int warp_search_with(const GraphView& g, DIST& dist, int32_t entry, i
         }
       }
     }
+    GANNS_PROF_MARK(kProfSort);
     // (6) candidate update: merge T into N keeping l entries
     int pmin = lp, nins = 0;
 #pragma unroll
@@ -886,7 +921,17 @@ __device__ int warp_search_with(const GraphView& g, DIST& dist, int32_t entry, i
     }
     cnt = ncnt;
     __syncwarp();
+    GANNS_PROF_MARK(kProfMerge);
   }
+#if GANNS_PROFILE
+  if (g.prof != nullptr && lane == 0) {
+#pragma unroll
+    for (int i = 0; i < 6; ++i) atomicAdd(g.prof + i, pc[i]);
+    atomicAdd(g.prof + 6, (unsigned long long)st.iters);
+    atomicAdd(g.prof + 7, 1ull);
+  }
+#endif
+#undef GANNS_PROF_MARK
   return cnt;
 }
 

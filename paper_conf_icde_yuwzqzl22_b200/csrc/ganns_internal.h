@@ -65,6 +65,8 @@ inline cudaError_t once_per_device(std::atomic<uint64_t>& done, F&& set) {
 // build: a cudaMalloc/cudaFree of the build scratch cost 2 ms typically and up to
 // 1 s of host time (profiles/r02/build_phases_host_gap.log), the pool 0.02 ms.
 cudaError_t pool_alloc(void** p, size_t bytes, cudaStream_t s);
+// GANNS_PROFILE builds: the current device's phase counters (8 x u64), else nullptr
+unsigned long long* prof_buffer();
 void pool_free(void* p, cudaStream_t s);
 
 void set_error(const std::string& msg);

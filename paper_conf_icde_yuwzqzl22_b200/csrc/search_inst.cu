@@ -212,6 +212,7 @@ static cudaError_t launch_t(const SearchLaunch& a, cudaStream_t s) {
     smem += size_t(pad);
   }
   GraphView g{a.nbr, a.X, nullptr, a.n, a.d_max, a.d / 4, a.metric};
+  g.prof = prof_buffer();
   CUtensorMap tmap;
   cudaError_t err = uses_tma(NV4) ? encode_row_tmap(a.X, a.n, a.d, &tmap) : zero_tmap(&tmap);
   if (err != cudaSuccess) return err;
@@ -303,6 +304,7 @@ static cudaError_t launch_group_t(const SearchLaunch& a, cudaStream_t s) {
   const size_t smem = smem_for(wrows);
   if (smem > 227 * 1024) return cudaErrorInvalidValue;
   GraphView g{a.nbr, a.X, nullptr, a.n, a.d_max, d4, a.metric};
+  g.prof = prof_buffer();
   cudaError_t err = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kGroupWarps * 32, smem);
   if (err != cudaSuccess) return err;
   int64_t blocks = a.nq;

@@ -88,3 +88,13 @@ def test_graph_load_rejects_corrupt_headers_before_allocating(tmp_path):
         h = ctypes.c_void_p()
         assert lib.ganns_graph_load(str(p).encode(), 0, ctypes.byref(h)) == -5, name
         assert h.value is None
+
+
+def test_profile_counters_need_a_profile_build():
+    """ganns_profile_read is GANNS_ENOTSUP (-4) in the normal build (the per-phase
+    timers are compiled in only with -DGANNS_PROFILE=1)."""
+    lib = ctypes.CDLL(LIB)
+    lib.ganns_profile_read.argtypes = [ctypes.c_void_p, ctypes.c_int]
+    lib.ganns_profile_read.restype = ctypes.c_int
+    out = (ctypes.c_uint64 * 8)()
+    assert lib.ganns_profile_read(ctypes.cast(out, ctypes.c_void_p), 0) == -4
