@@ -331,6 +331,14 @@ GANNS_API uint64_t ganns_kernel_launches(void);
  * -DGANNS_PROFILE=1 (tools/build_variants.sh prof -DGANNS_PROFILE=1). */
 GANNS_API int ganns_profile_read(uint64_t *out, int reset);
 
+/* ganns_profile_read_n -- the same counters, `count` (0..16) of them: out[0..7] as
+ * above; inside the bulk distance out[8] = cycles from the start of a TMA round to
+ * its last issue, out[9] = cycles waiting on the round's mbarrier, out[10] = TMA
+ * rounds; out[11] = explorations whose adjacency row the speculative load of the
+ * second unexplored entry had already fetched; out[12] / out[13] = the largest loop
+ * cycles / iterations of a single search (maxima).  GANNS_EINVAL if count is out of range. */
+GANNS_API int ganns_profile_read_n(uint64_t *out, int count, int reset);
+
 #ifdef __cplusplus
 }
 #endif

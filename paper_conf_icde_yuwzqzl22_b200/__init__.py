@@ -93,6 +93,8 @@ def _load():
     lib.ganns_kernel_launches.restype = ct.c_uint64
     lib.ganns_profile_read.argtypes = [P, i32]
     lib.ganns_profile_read.restype = ct.c_int
+    lib.ganns_profile_read_n.argtypes = [P, i32, i32]
+    lib.ganns_profile_read_n.restype = ct.c_int
     return lib
 
 
@@ -109,7 +111,7 @@ ABI_SYMBOLS = ("ganns_build", "ganns_search", "ganns_search_ex", "ganns_search_h
                "ganns_hnsw_free", "ganns_build_knn", "ganns_build_begin", "ganns_build_info",
                "ganns_build_phase1", "ganns_build_rows", "ganns_build_round_search",
                "ganns_build_round_apply", "ganns_build_finish", "ganns_build_abort",
-               "ganns_profile_read")
+               "ganns_profile_read", "ganns_profile_read_n")
 
 
 def lib():
@@ -176,10 +178,13 @@ PROFILE_PHASES = ("locate", "explore", "distance", "lazy_check", "sort", "merge"
 def profile_read(reset: bool = True):
     """Per-phase cycle counters of a GANNS_PROFILE library build (ganns_profile_read):
     dict(phase -> cycles, iterations, searches).  Raises on a normal build."""
-    out = (ct.c_uint64 * 8)()
-    _check(_lib.ganns_profile_read(ct.cast(out, ct.c_void_p), int(reset)))
+    out = (ct.c_uint64 * 14)()
+    _check(_lib.ganns_profile_read_n(ct.cast(out, ct.c_void_p), 14, int(reset)))
     d = {k: int(out[i]) for i, k in enumerate(PROFILE_PHASES)}
     d["iterations"], d["searches"] = int(out[6]), int(out[7])
+    d["gather_issue"], d["gather_wait"], d["gather_rounds"] = int(out[8]), int(out[9]), int(out[10])
+    d["spec_hits"] = int(out[11])
+    d["max_search_cycles"], d["max_search_iterations"] = int(out[12]), int(out[13])
     return d
 
 

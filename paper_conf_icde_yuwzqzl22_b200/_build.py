@@ -85,5 +85,31 @@ def build(force: bool = False, verbose: bool = False) -> str:
     return LIB
 
 
+def build_variant(out: str, defines: list[str], dev: bool = True) -> str:
+    """A/B and profiling variants (tools/): the library with extra -D flags, linked to
+    `out`, objects in their own directory; the default library is untouched.
+    dev=True compiles only the d <= 128 / d_max <= 32 instances (the DEV_UNITS)."""
+    tag = os.path.splitext(os.path.basename(out))[0]
+    odir = os.path.join(OBJ, "var_" + tag)
+    os.makedirs(odir, exist_ok=True)
+    units = [(src, defs + defines, obj) for src, defs, obj in (DEV_UNITS if dev else UNITS)]
+
+    def comp(u):
+        src, defs, obj = u
+        o = os.path.join(odir, obj)
+        r = subprocess.run([NVCC, *ARCH, *FLAGS, *defs, "-c", os.path.join(CSRC, src), "-o", o],
+                           capture_output=True, text=True)
+        if r.returncode != 0:
+            raise RuntimeError(f"nvcc failed for {src} {defs}:\n{r.stderr}")
+        return o
+    with cf.ThreadPoolExecutor(max_workers=max(2, min(len(units), os.cpu_count() or 2))) as ex:
+        objs = list(ex.map(comp, units))
+    os.makedirs(os.path.dirname(os.path.abspath(out)), exist_ok=True)
+    r = subprocess.run([NVCC, *ARCH, "-shared", "-o", out, *objs, "-lcudart"], capture_output=True, text=True)
+    if r.returncode != 0:
+        raise RuntimeError(f"link failed:\n{r.stderr}")
+    return out
+
+
 if __name__ == "__main__":
     build(force=True, verbose=True)

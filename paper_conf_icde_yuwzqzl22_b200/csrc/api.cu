@@ -52,8 +52,8 @@ unsigned long long* prof_buffer() {
   if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return nullptr;
   std::lock_guard<std::mutex> lock(mu);
   if (!buf[dev]) {
-    if (cudaMalloc(&buf[dev], 8 * sizeof(unsigned long long)) != cudaSuccess) return nullptr;
-    cudaMemset(buf[dev], 0, 8 * sizeof(unsigned long long));
+    if (cudaMalloc(&buf[dev], kProfSlots * sizeof(unsigned long long)) != cudaSuccess) return nullptr;
+    cudaMemset(buf[dev], 0, kProfSlots * sizeof(unsigned long long));
   }
   return buf[dev];
 #else
@@ -210,15 +210,18 @@ extern "C" {
 const char* ganns_last_error(void) { return g_last_error.c_str(); }
 uint64_t ganns_kernel_launches(void) { return g_launches.load(); }
 
-int ganns_profile_read(uint64_t* out, int reset) {
+int ganns_profile_read_n(uint64_t* out, int count, int reset) {
   unsigned long long* p = prof_buffer();
   if (!p) return fail(GANNS_ENOTSUP, "library built without GANNS_PROFILE");
   if (!out) return fail(GANNS_EINVAL, "out is NULL");
+  if (count < 0 || count > kProfSlots) return fail(GANNS_EINVAL, "count out of range");
   cudaError_t e = cudaDeviceSynchronize();
-  if (e == cudaSuccess) e = cudaMemcpy(out, p, 8 * sizeof(uint64_t), cudaMemcpyDeviceToHost);
-  if (e == cudaSuccess && reset) e = cudaMemset(p, 0, 8 * sizeof(uint64_t));
+  if (e == cudaSuccess) e = cudaMemcpy(out, p, size_t(count) * sizeof(uint64_t), cudaMemcpyDeviceToHost);
+  if (e == cudaSuccess && reset) e = cudaMemset(p, 0, kProfSlots * sizeof(uint64_t));
   return e == cudaSuccess ? GANNS_OK : cuda_fail(e, "ganns_profile_read");
 }
+
+int ganns_profile_read(uint64_t* out, int reset) { return ganns_profile_read_n(out, 8, reset); }
 
 int ganns_graph_info(const ganns_graph* g, int64_t* n, int* d, int* d_max, int* metric) {
   if (int rc = check_graph(g)) return rc;

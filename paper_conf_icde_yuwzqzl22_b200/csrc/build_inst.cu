@@ -53,6 +53,50 @@ constexpr int kBuildWarps = 1;   // one warp per CTA spreads the latency-bound b
 // warp-min and load sit on the chain and the hidden adjacency latency is small (the
 // adjacency rows mostly hit L2)
 constexpr bool kBuildPredict = GANNS_BUILD_PREDICT != 0;
+// The build searches' stage is filled by cp.async (ganns_dev.cuh: cpasync_fill) for
+// d <= 256, and (d_max <= 32) the next exploration's rows are gathered
+// speculatively while the lazy check, sort and merge run (warp_search_with, SPEC).
+// A build search is a latency chain: a Phase-2 round lasts as long as its slowest
+// search (1.05x, tools/round_tail.py), which runs 1.7x the mean iteration count.
+#ifndef GANNS_BUILD_CPASYNC
+#define GANNS_BUILD_CPASYNC 1
+#endif
+#ifndef GANNS_BUILD_SPEC
+#define GANNS_BUILD_SPEC 1
+#endif
+template <int NV4>
+constexpr bool kBuildCpAsync = GANNS_BUILD_CPASYNC != 0 && uses_tma(NV4);
+template <int NV4, int TPL>
+constexpr bool kBuildSpec = GANNS_BUILD_SPEC != 0 && kBuildCpAsync<NV4> && TPL == 1 && !kBuildPredict;
+// GANNS_BUILD_P1: Phase 1 (l_local searches on the local graphs) uses the same
+// cp.async + speculation form as Phase 2; else the TMA tile::gather4 form
+#ifndef GANNS_BUILD_P1
+#define GANNS_BUILD_P1 1
+#endif
+template <int NV4>
+constexpr bool kP1CpAsync = kBuildCpAsync<NV4> && GANNS_BUILD_P1 != 0;
+template <int NV4, int TPL>
+constexpr bool kP1Spec = kBuildSpec<NV4, TPL> && GANNS_BUILD_P1 != 0;
+#ifndef GANNS_BUILD_T_OUT
+#define GANNS_BUILD_T_OUT 1
+#endif
+
+// Per-warp shared memory of a build search: the search's area, then (cp.async
+// form) T outside the stage
+template <int NV4, int TPL>
+__host__ __device__ constexpr size_t build_warp_bytes(int l, int d4) {
+  return warp_smem_bytes(l, TPL, NV4, d4, kBuildStageRounds) +
+         (kBuildCpAsync<NV4> && GANNS_BUILD_T_OUT ? t_bytes(TPL) : 0);
+}
+template <int NV4, int TPL>
+__device__ __forceinline__ WarpSmem carve_build_smem(uint8_t* smem, int w, int l, int d4) {
+  uint8_t* base = smem + size_t(w) * build_warp_bytes<NV4, TPL>(l, d4);
+  WarpSmem ws = carve_warp_smem(base, l, TPL, NV4, d4, kBuildStageRounds);
+  if constexpr (kBuildCpAsync<NV4> && GANNS_BUILD_T_OUT) {
+    ws.sT = reinterpret_cast<uint64_t*>(base + warp_smem_bytes(l, TPL, NV4, d4, kBuildStageRounds));
+  }
+  return ws;
+}
 
 // Insert key kx into a warp-distributed ascending row of d_max keys (TPL per
 // lane, slot j = t*32 + lane); the last key falls off when the row is full
@@ -137,9 +181,7 @@ phase1_kernel(BuildDev B, int64_t group_size, int64_t g0, int64_t g1,
   const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int64_t gi = g0 + int64_t(blockIdx.x) * kBuildWarps + w;   // groups [g0, g1)
   if (gi >= g1) return;
-  WarpSmem ws = carve_warp_smem(
-      smem + size_t(w) * warp_smem_bytes(B.l_build, TPL, NV4, B.g.d4, kBuildStageRounds),
-      B.l_build, TPL, NV4, B.g.d4, kBuildStageRounds);
+  WarpSmem ws = carve_build_smem<NV4, TPL>(smem, w, B.l_build, B.g.d4);
   if (lane == 0) mbar_init(ws.mbar, 1);
   __syncwarp();
   uint64_t* sN = ws.sN;
@@ -149,8 +191,8 @@ phase1_kernel(BuildDev B, int64_t group_size, int64_t g0, int64_t g1,
   for (int64_t v = lo + 1; v < hi; ++v) {
     // Step 1 (line 5): v.N, v.N' := Search(G_i, v, d_min), entry = group's first vertex
     SearchStats st;
-    const int cnt = warp_search<NV4, TPL, L2, true, kBuildPredict>(B.g, B.g.X + size_t(v) * d, int32_t(lo),
-                                                    B.l_local, B.e_local, ws, st);
+    const int cnt = warp_search<NV4, TPL, L2, true, kBuildPredict, kP1Spec<NV4, TPL>, kP1CpAsync<NV4>>(
+        B.g, B.g.X + size_t(v) * d, int32_t(lo), B.l_local, B.e_local, ws, st);
     add_stats(B.stats, st, lane);
     const int m = cnt < B.d_min ? cnt : B.d_min;
     for (int j = lane; j < m; j += 32) {
@@ -192,7 +234,9 @@ phase1_kernel(BuildDev B, int64_t group_size, int64_t g0, int64_t g1,
 // (multi-GPU build): only the new forward row F (first d_min) is written, to
 // F_ids / F_dists [(v - v0)][d_min]; apply_forward_kernel consumes the F of all of
 // P_i after the exchange.
-template <int NV4, int TPL, bool L2>
+// HNSW: the instance that enters through the descent of the upper layers (the
+// plain NSW build's instance carries no descent code)
+template <int NV4, int TPL, bool L2, bool HNSW>
 __global__ void __launch_bounds__(kBuildWarps * 32)
 round_search_kernel(BuildDev B, int64_t lo, int64_t v0, int64_t v1, int32_t* __restrict__ Eu,
                     float* __restrict__ Ed, int32_t* __restrict__ indeg,
@@ -204,9 +248,7 @@ round_search_kernel(BuildDev B, int64_t lo, int64_t v0, int64_t v1, int32_t* __r
   const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int64_t v = v0 + int64_t(blockIdx.x) * kBuildWarps + w;
   if (v >= v1) return;
-  WarpSmem ws = carve_warp_smem(
-      smem + size_t(w) * warp_smem_bytes(B.l_build, TPL, NV4, B.g.d4, kBuildStageRounds),
-      B.l_build, TPL, NV4, B.g.d4, kBuildStageRounds);
+  WarpSmem ws = carve_build_smem<NV4, TPL>(smem, w, B.l_build, B.g.d4);
   if (lane == 0) mbar_init(ws.mbar, 1);
   __syncwarp();
   uint64_t* sN = ws.sN;
@@ -216,13 +258,16 @@ round_search_kernel(BuildDev B, int64_t lo, int64_t v0, int64_t v1, int32_t* __r
   // HNSW: enter through a greedy descent of the finished upper layers,
   // kept only if the vertex reached is already in G_0 (R-H2)
   int32_t entry = 0;
-  if (U.top > layer) {
-    const int32_t c = descend<NV4, TPL, L2>(B.g, U, layer + 1, B.g.X + size_t(v) * d, ws);
-    entry = c < lo ? c : 0;
+  if constexpr (HNSW) {
+    if (U.top > layer) {
+      const int32_t c = descend<NV4, TPL, L2, kBuildCpAsync<NV4>>(B.g, U, layer + 1,
+                                                                 B.g.X + size_t(v) * d, ws);
+      entry = c < lo ? c : 0;
+    }
   }
   SearchStats st;
-  const int cnt = warp_search<NV4, TPL, L2, false, kBuildPredict>(B.g, B.g.X + size_t(v) * d, entry, B.l_build,
-                                                   B.e_build, ws, st);
+  const int cnt = warp_search<NV4, TPL, L2, false, kBuildPredict, kBuildSpec<NV4, TPL>, kBuildCpAsync<NV4>>(
+      B.g, B.g.X + size_t(v) * d, entry, B.l_build, B.e_build, ws, st);
   add_stats(B.stats, st, lane);
   const int dm = B.d_min;
   const int cs = cnt < dm ? cnt : dm;
@@ -395,7 +440,10 @@ static cudaError_t set_smem_attrs() {
     cudaError_t e = cudaFuncSetAttribute(phase1_kernel<NV4, TPL, L2>,
                                          cudaFuncAttributeMaxDynamicSharedMemorySize, mx);
     if (e == cudaSuccess)
-      e = cudaFuncSetAttribute(round_search_kernel<NV4, TPL, L2>,
+      e = cudaFuncSetAttribute(round_search_kernel<NV4, TPL, L2, false>,
+                               cudaFuncAttributeMaxDynamicSharedMemorySize, mx);
+    if (e == cudaSuccess)
+      e = cudaFuncSetAttribute(round_search_kernel<NV4, TPL, L2, true>,
                                cudaFuncAttributeMaxDynamicSharedMemorySize, mx);
     return e;
   });
@@ -443,10 +491,15 @@ static int round_search_t(BuildState& st, int64_t i, int64_t v0, int64_t v1, int
   if (v1 <= v0) return 0;
   if (f_ids == nullptr)   // fused form: counters of this round's GatherScatter start at 0
     GANNS_TRY(cudaMemsetAsync(st.counters, 0, sizeof(int32_t) * 2, s));
-  round_search_kernel<NV4, TPL, L2><<<unsigned((v1 - v0 + kBuildWarps - 1) / kBuildWarps),
-                                      kBuildWarps * 32, ds->smem, s>>>(
-      ds->B, lo, v0, v1, st.Eu, st.Ed, st.indeg, st.touched, st.counters, f_ids, f_dists, st.tmap,
-      ds->U, st.a.layer);
+  const unsigned grid = unsigned((v1 - v0 + kBuildWarps - 1) / kBuildWarps);
+  if (ds->U.top > st.a.layer)
+    round_search_kernel<NV4, TPL, L2, true><<<grid, kBuildWarps * 32, ds->smem, s>>>(
+        ds->B, lo, v0, v1, st.Eu, st.Ed, st.indeg, st.touched, st.counters, f_ids, f_dists, st.tmap,
+        ds->U, st.a.layer);
+  else
+    round_search_kernel<NV4, TPL, L2, false><<<grid, kBuildWarps * 32, ds->smem, s>>>(
+        ds->B, lo, v0, v1, st.Eu, st.Ed, st.indeg, st.touched, st.counters, f_ids, f_dists, st.tmap,
+        ds->U, st.a.layer);
   count_launch();
   GANNS_TRY(cudaGetLastError());
   return 0;
@@ -535,7 +588,7 @@ static int begin_t(BuildState& st, cudaStream_t s) {
   B.l_local = a.l_local > 0 ? a.l_local : a.l_build;
   B.e_local = a.e_local > 0 ? a.e_local : a.e_build;
   B.stats = st.stats;
-  ds->smem = size_t(kBuildWarps) * warp_smem_bytes(a.l_build, TPL, NV4, a.d / 4, kBuildStageRounds);
+  ds->smem = size_t(kBuildWarps) * build_warp_bytes<NV4, TPL>(a.l_build, a.d / 4);
   if (ds->smem > 227 * 1024) return fail(GANNS_ENOTSUP, "build: shared memory per CTA exceeds 227 KB");
   ds->U.top = a.upper.top;
   for (int j = 0; j < kMaxLayers; ++j) {

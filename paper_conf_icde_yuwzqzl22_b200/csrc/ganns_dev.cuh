@@ -148,11 +148,16 @@ struct GraphView {
 // (a separate library build): lane 0 of each warp reads clock64() at the phase
 // boundaries and adds the cycles to prof[0..5] = candidate locating, neighbourhood
 // exploration (adjacency row), bulk distance (gather + math), lazy check, sort,
-// merge; prof[6] = iterations, prof[7] = searches.
+// merge; prof[6] = iterations, prof[7] = searches; inside the bulk distance
+// prof[8] = cycles from the start of a gather to its last TMA issue, prof[9] =
+// cycles waiting on the gather's mbarrier, prof[10] = TMA rounds; prof[11] =
+// explorations whose adjacency row the speculation had already loaded; prof[12] /
+// prof[13] = the largest cycles / iterations of one search (max, not sum).
 #ifndef GANNS_PROFILE
 #define GANNS_PROFILE 0
 #endif
 enum { kProfLocate = 0, kProfExplore, kProfDistance, kProfLazy, kProfSort, kProfMerge };
+
 
 // Per-search counters (kept in registers, identical to the oracle's stats[0,1,3]).
 struct SearchStats {
@@ -249,6 +254,9 @@ struct WarpSmem {
   float4* pair_stage;
   volatile int* pair_flag;
   int pair_bar;   // named barrier of the pair (64 threads): leaver arrives, taker syncs
+#if GANNS_PROFILE
+  unsigned long long p_issue = 0, p_wait = 0, p_rounds = 0;   // lane 0's gather timers
+#endif
 };
 // Per-CTA layout of the pooled search kernel: [pool stages][per-warp N/T/bitmap][pool meta]
 __host__ __device__ constexpr size_t pooled_warp_bytes(int l, int tpl) {
@@ -417,6 +425,9 @@ __device__ __forceinline__ float tma_dot(const GraphView& g, const float4 (&qv)[
   stage_acquire(ws, lane);
 #pragma unroll
   for (int r = 0; r < ROUNDS; ++r) {
+#if GANNS_PROFILE
+    const long long t_g0 = clock64();
+#endif
     // tile::gather4 (d % 8 == 0, so every group of 4 rows starts 128-B aligned):
     // lane 4m of this round fetches the rows of lanes 4m..4m+3 into 4 consecutive
     // stage slots with ONE TMA instruction; absent neighbours get an out-of-range
@@ -460,8 +471,17 @@ __device__ __forceinline__ float tma_dot(const GraphView& g, const float4 (&qv)[
           tma_row(dst, reinterpret_cast<const char*>(g.X) + uint64_t(uint32_t(u_mine)) * rowbytes,
                   rowbytes, ws.mbar);
       }
+#if GANNS_PROFILE
+      const long long t_g1 = clock64();
+#endif
       mbar_wait(ws.mbar, ws.phase);
       ws.phase ^= 1u;
+#if GANNS_PROFILE
+      const long long t_g2 = clock64();
+      ws.p_issue += t_g1 - t_g0;
+      ws.p_wait += t_g2 - t_g1;
+      ws.p_rounds += 1;
+#endif
     }
 #pragma unroll
     for (int gg = 0; gg < PPR; ++gg) {
@@ -477,6 +497,105 @@ __device__ __forceinline__ float tma_dot(const GraphView& g, const float4 (&qv)[
     }
   }
   stage_release(ws, lane);
+#pragma unroll
+  for (int half = S / 2; half >= 1; half >>= 1) {
+    const bool up = lane & half;
+#pragma unroll
+    for (int i = 0; i < half; ++i) {
+      float send = up ? p[i] : p[i + half];
+      float keep = up ? p[i + half] : p[i];
+      p[i] = keep + __shfl_xor_sync(kFull, send, half);
+    }
+  }
+  return p[0];
+}
+
+// One-round segment form with the stage filled by per-lane async copies
+// (cp.async.cg, SASS LDGSTS: 16 B per lane, one warp instruction per 512 B of a
+// row, L2 only) instead of TMA -- the form of the build searches (ws.cpasync).
+// The row of lane L goes to slot L as in tma_dot's one-round layout, so the math
+// is the same.  Rows are copied in pass order in two commit groups: the first
+// half of the passes starts its math while the second half's rows still arrive.
+// No mbarrier and no uniform-register issue loop (a tile::gather4 per 4 rows
+// costs one ELECT / R2UR waterfall iteration per issuing lane), and no proxy
+// fence: cp.async writes are generic-proxy writes.
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
+// 16 B of row u (u >= 0; else nothing) at byte offset `src` of the rows' base
+// (the lane's chunk) -> shared address dst: one predicate, one address, one copy
+__device__ __forceinline__ void cp_async_row16(uint32_t dst, const void* src, int32_t u,
+                                               uint32_t rowbytes) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t.reg .u64 a;\n\tsetp.ge.s32 p, %2, 0;\n\t"
+      "mad.wide.u32 a, %2, %3, %1;\n\t@p cp.async.cg.shared.global [%0], [a], 16;\n\t}" ::"r"(dst),
+      "l"(src), "r"(u), "r"(rowbytes)
+      : "memory");
+}
+
+// issue the copies of the <= 32 rows (u_mine per lane, -1 = none) into the stage:
+// one warp instruction per 512 B of a row (lane c copies 16-B chunk c, and c + 32
+// for d > 128), straight-line and predicated -- per row a shuffle of its id, a
+// predicate, an address and the copy (a branchy per-row loop cost ~18
+// instructions per row and instruction-cache misses); two commit groups (the rows
+// of passes [0, S/2), then [S/2, S)).  FULL: d = 4 * S * C, the row size is a
+// compile-time constant (the stage offsets become immediates).
+template <int S, bool FULL>
+__device__ __forceinline__ void cpasync_fill(const GraphView& g, int32_t u_mine, int lane,
+                                             const WarpSmem& ws) {
+  constexpr int NSEG = 32 / S;
+  constexpr int CH = S / 8;   // 16-B chunks per lane per row: d <= 128 -> 1, d <= 256 -> 2
+  const uint32_t rowbytes = FULL ? uint32_t(S) * 64u : uint32_t(g.d4) * 16u;
+  const uint32_t sbase = smem_u32(ws.stage) + uint32_t(lane) * 16u;
+  const char* xb = reinterpret_cast<const char*>(g.X) + lane * 16;
+  bool in[CH];
+#pragma unroll
+  for (int j = 0; j < CH; ++j) in[j] = FULL || lane + 32 * j < g.d4;
+#pragma unroll
+  for (int gg = 0; gg < S; ++gg) {
+#pragma unroll
+    for (int s = 0; s < NSEG; ++s) {
+      const int L = gg + S * s;
+      const int32_t u = __shfl_sync(kFull, u_mine, L);
+#pragma unroll
+      for (int j = 0; j < CH; ++j)
+        cp_async_row16(sbase + uint32_t(L) * rowbytes + 512u * j, xb + 512 * j, in[j] ? u : -1,
+                       rowbytes);
+    }
+    if (gg == S / 2 - 1) cp_async_commit();
+  }
+  cp_async_commit();
+}
+
+// the math over a stage filled by cpasync_fill (its two groups must be this
+// thread's last two commits; any older group is waited for as well)
+template <int S, int C, bool L2, bool FULL>
+__device__ __forceinline__ float cpasync_math(const GraphView& g, const float4 (&qv)[C], int lane,
+                                              WarpSmem& ws) {
+  const int sl = lane & (S - 1), seg = lane / S;
+  int coff[C];
+#pragma unroll
+  for (int f = 0; f < C; ++f) coff[f] = (FULL || sl + S * f < g.d4) ? sl + S * f : g.d4 - 1;
+  float p[S];
+#pragma unroll
+  for (int gg = 0; gg < S; ++gg) {
+    if (gg == 0) {
+      cp_async_wait<1>();
+      __syncwarp();
+    } else if (gg == S / 2) {
+      cp_async_wait<0>();
+      __syncwarp();
+    }
+    const float4* rp = ws.stage + size_t(gg + S * seg) * g.d4;
+    float4 x[C];
+#pragma unroll
+    for (int f = 0; f < C; ++f) x[f] = lds128_ordered(rp + coff[f]);
+    uint64_t acc = 0;
+#pragma unroll
+    for (int f = 0; f < C; ++f)
+      if (FULL || sl + S * f < g.d4) acc = accum4<L2>(acc, qv[f], x[f]);
+    p[gg] = hsum2(acc);
+  }
 #pragma unroll
   for (int half = S / 2; half >= 1; half >>= 1) {
     const bool up = lane & half;
@@ -555,7 +674,9 @@ __device__ __forceinline__ float wide_dot(const GraphView& g, const float4 (&qv)
   return dres;
 }
 
-template <int NV4, bool L2>
+// CPA (build searches, d <= 256): the stage is filled by cp.async (cpasync_fill),
+// one round of <= 32 rows
+template <int NV4, bool L2, bool CPA = false>
 __device__ __forceinline__ float group_distances(const GraphView& g,
                                                  const float4 (&qv)[VecLayout<NV4>::C],
                                                  int32_t u_mine, float cbase, float qinv,
@@ -565,7 +686,15 @@ __device__ __forceinline__ float group_distances(const GraphView& g,
   const bool full = g.d4 == S * C;
   float dot;
   if constexpr (S < 32) {
-    if (ws.rounds == 1)
+    if constexpr (CPA) {
+      if (full) {
+        cpasync_fill<S, true>(g, u_mine, lane, ws);
+        dot = cpasync_math<S, C, L2, true>(g, qv, lane, ws);
+      } else {
+        cpasync_fill<S, false>(g, u_mine, lane, ws);
+        dot = cpasync_math<S, C, L2, false>(g, qv, lane, ws);
+      }
+    } else if (ws.rounds == 1)
       dot = full ? tma_dot<S, C, L2, true, 1>(g, qv, u_mine, lane, ws)
                  : tma_dot<S, C, L2, false, 1>(g, qv, u_mine, lane, ws);
 #if GANNS_SEARCH_ROUNDS == 4
@@ -587,8 +716,9 @@ __device__ __forceinline__ float group_distances(const GraphView& g,
 
 // Bulk-distance policy of one warp (the default): the query slice lives in this
 // warp's registers and the warp computes all distances of an exploration itself.
-template <int NV4, bool L2>
+template <int NV4, bool L2, bool CPA = false>
 struct WarpDist {
+  static_assert(!CPA || uses_tma(NV4), "the cp.async form is the segment form (d <= 256)");
   static constexpr int S = VecLayout<NV4>::S, C = VecLayout<NV4>::C;
   float4 qv[C];
   float cbase, qinv;
@@ -624,6 +754,22 @@ struct WarpDist {
         prefetch_row_l2(g.X + size_t(u_mine) * (g.d4 * 4), uint32_t(g.d4) * 16u);
 #endif
   }
+  // SPEC (build searches, CPA): the gather of an exploration's rows is
+  // issued by fill() -- possibly one iteration early -- and reduced by math()
+  __device__ __forceinline__ void fill(const GraphView& g, int32_t u_mine, int lane, WarpSmem& ws) {
+    if constexpr (uses_tma(NV4)) {
+      if (g.d4 == S * C) cpasync_fill<S, true>(g, u_mine, lane, ws);
+      else cpasync_fill<S, false>(g, u_mine, lane, ws);
+    }
+  }
+  __device__ __forceinline__ float math(const GraphView& g, int lane, WarpSmem& ws) {
+    float dot = 0.f;
+    if constexpr (uses_tma(NV4))
+      dot = g.d4 == S * C ? cpasync_math<S, C, L2, true>(g, qv, lane, ws)
+                          : cpasync_math<S, C, L2, false>(g, qv, lane, ws);
+    if constexpr (L2) return dot;
+    else return cbase - dot * qinv;
+  }
   __device__ __forceinline__ float operator()(const GraphView& g, int32_t u_mine, int lane,
                                               WarpSmem& ws) {
     if constexpr (uses_tma(NV4))
@@ -639,7 +785,7 @@ struct WarpDist {
           ws.stage = ws.pair_stage;
         }
       }
-    return group_distances<NV4, L2>(g, qv, u_mine, cbase, qinv, lane, ws);
+    return group_distances<NV4, L2, CPA>(g, qv, u_mine, cbase, qinv, lane, ws);
   }
 };
 
@@ -652,9 +798,18 @@ struct WarpDist {
 // predicted -- the smallest surviving neighbour always enters N, so it is next
 // whenever it precedes the second unexplored entry w -- and its adjacency row is
 // loaded while the sort and merge run.  Results never depend on the prediction.
-template <class DIST, int TPL, bool COHERENT, bool PREDICT = false>
+// SPEC (build searches with ws.cpasync, d_max <= 32): right after an exploration's
+// distance math, the rows of w (the second unexplored entry, whose adjacency row
+// the speculation loads with v's) are gathered into the stage -- the stage is
+// idle during the lazy check, sort and merge (T lives outside it).  When w is
+// the next vertex explored (2/3 to 4/5 of the iterations in the C2 build), its
+// rows have arrived meanwhile; otherwise the copies are drained and the right
+// rows gathered.  Results never depend on the speculation.
+template <class DIST, int TPL, bool COHERENT, bool PREDICT = false, bool SPEC = false>
 __device__ int warp_search_with(const GraphView& g, DIST& dist, int32_t entry, int l, int e,
                                 WarpSmem& ws, SearchStats& st) {
+  static_assert(!(SPEC && PREDICT), "one speculation at a time");
+  static_assert(!SPEC || TPL == 1, "SPEC gathers one 32-row round");
   const int lane = threadIdx.x & 31;
   uint64_t* sN = ws.sN;
   uint64_t* sT = ws.sT;
@@ -684,8 +839,11 @@ __device__ int warp_search_with(const GraphView& g, DIST& dist, int32_t entry, i
   int32_t spec_u[TPL];
   int32_t pred_v = -1;      // PREDICT: the vertex predicted after the last lazy check
   int32_t pred_u[TPL];
+  int32_t gath_v = -1;      // SPEC: the vertex whose neighbours' rows are in the stage
 #if GANNS_PROFILE
   unsigned long long pc[6] = {0, 0, 0, 0, 0, 0};
+  unsigned long long p_spec = 0;
+  ws.p_issue = ws.p_wait = ws.p_rounds = 0;
   long long tp = clock64();
 #define GANNS_PROF_MARK(i)          \
   {                                 \
@@ -739,6 +897,7 @@ __device__ int warp_search_with(const GraphView& g, DIST& dist, int32_t entry, i
     spec_v = w;
     pred_v = -1;
 #if GANNS_PROFILE
+    p_spec += hit ? 1 : 0;
     if (__ballot_sync(kFull, u[0] >= 0) == 0xdeadbeefu) st.merged += 0;   // waits for the row
     GANNS_PROF_MARK(kProfExplore);
 #endif
@@ -746,11 +905,47 @@ __device__ int warp_search_with(const GraphView& g, DIST& dist, int32_t entry, i
 #pragma unroll
     for (int t = 0; t < TPL; ++t) dist.explore_hint(g, u[t], lane, ws);
     uint64_t key[TPL];
+    if constexpr (SPEC) {
+#if GANNS_PROFILE
+      // SPEC timers: p_issue = cycles issuing copies (both fills), p_wait = the
+      // math incl. its waits, p_rounds = explorations whose rows were gathered ahead
+      const long long t_s0 = clock64();
+      ws.p_rounds += v == gath_v ? 1 : 0;
+#endif
+      if (v != gath_v) {   // not gathered ahead: drain the speculative copies, gather
+        if (gath_v >= 0) {
+          cp_async_wait<0>();
+          __syncwarp();
+        }
+        dist.fill(g, u[0], lane, ws);
+      }
+#if GANNS_PROFILE
+      const long long t_s1 = clock64();
+#endif
+      const float dd = dist.math(g, lane, ws);
+      key[0] = u[0] >= 0 ? mkkey(dd, u[0]) : kKeyInf;
+      st.comps += __popc(__ballot_sync(kFull, u[0] >= 0));
+      __syncwarp();   // every lane's stage reads precede the next copies into it
+#if GANNS_PROFILE
+      const long long t_s2 = clock64();
+#endif
+      gath_v = -1;
+      if (w >= 0) {   // spec_u = w's adjacency row (loaded with v's)
+        dist.fill(g, spec_u[0], lane, ws);
+        gath_v = w;
+      }
+#if GANNS_PROFILE
+      const long long t_s3 = clock64();
+      ws.p_issue += (t_s1 - t_s0) + (t_s3 - t_s2);
+      ws.p_wait += t_s2 - t_s1;
+#endif
+    } else {
 #pragma unroll
-    for (int t = 0; t < TPL; ++t) {
-      float dd = dist(g, u[t], lane, ws);
-      key[t] = u[t] >= 0 ? mkkey(dd, u[t]) : kKeyInf;
-      st.comps += __popc(__ballot_sync(kFull, u[t] >= 0));
+      for (int t = 0; t < TPL; ++t) {
+        float dd = dist(g, u[t], lane, ws);
+        key[t] = u[t] >= 0 ? mkkey(dd, u[t]) : kKeyInf;
+        st.comps += __popc(__ballot_sync(kFull, u[t] >= 0));
+      }
     }
     __syncwarp();   // every lane's stage reads precede the merge's writes of T (it shares the stage)
     GANNS_PROF_MARK(kProfDistance);
@@ -913,7 +1108,8 @@ __device__ int warp_search_with(const GraphView& g, DIST& dist, int32_t entry, i
         __syncwarp();
       }
 #if GANNS_LATE_FENCE
-      fence_proxy_async_smem();   // T's generic writes (in the stage) precede the next TMA writes
+      if constexpr (!SPEC)
+        fence_proxy_async_smem();   // T's generic writes (in the stage) precede the next TMA writes
 #endif
       hint = pmin < found + 1 ? pmin : found + 1;
     } else {
@@ -923,25 +1119,43 @@ __device__ int warp_search_with(const GraphView& g, DIST& dist, int32_t entry, i
     __syncwarp();
     GANNS_PROF_MARK(kProfMerge);
   }
+  if constexpr (SPEC)
+    if (gath_v >= 0) {   // the last speculation's copies land before the stage is reused
+      cp_async_wait<0>();
+      __syncwarp();
+    }
 #if GANNS_PROFILE
   if (g.prof != nullptr && lane == 0) {
 #pragma unroll
     for (int i = 0; i < 6; ++i) atomicAdd(g.prof + i, pc[i]);
     atomicAdd(g.prof + 6, (unsigned long long)st.iters);
     atomicAdd(g.prof + 7, 1ull);
+    atomicAdd(g.prof + 8, ws.p_issue);
+    atomicAdd(g.prof + 9, ws.p_wait);
+    atomicAdd(g.prof + 10, ws.p_rounds);
+    atomicAdd(g.prof + 11, p_spec);
+    unsigned long long tot = 0;
+#pragma unroll
+    for (int i = 0; i < 6; ++i) tot += pc[i];
+    atomicMax(g.prof + 12, tot);
+    atomicMax(g.prof + 13, (unsigned long long)st.iters);
   }
 #endif
 #undef GANNS_PROF_MARK
   return cnt;
 }
 
-template <int NV4, int TPL, bool L2, bool COHERENT, bool PREDICT = false>
+// CPA: the build searches' cp.async gathers (group_distances); SPEC requires it
+template <int NV4, int TPL, bool L2, bool COHERENT, bool PREDICT = false, bool SPEC = false,
+          bool CPA = SPEC>
 __device__ __forceinline__ int warp_search(const GraphView& g, const float* __restrict__ qrow,
                                            int32_t entry, int l, int e, WarpSmem& ws,
                                            SearchStats& st) {
-  WarpDist<NV4, L2> dist;
+  static_assert(!SPEC || CPA, "the speculative gather is a cp.async gather");
+  WarpDist<NV4, L2, CPA> dist;
   dist.load(g, qrow, threadIdx.x & 31);
-  return warp_search_with<WarpDist<NV4, L2>, TPL, COHERENT, PREDICT>(g, dist, entry, l, e, ws, st);
+  return warp_search_with<WarpDist<NV4, L2, CPA>, TPL, COHERENT, PREDICT, SPEC>(g, dist, entry, l, e,
+                                                                               ws, st);
 }
 
 // ---------------------------------------------------------------- HNSW
@@ -957,6 +1171,14 @@ struct UpperLayers {
 // Greedy descent: the GANNS search with l = e = 1 (the best candidate only) from
 // shuffled id 0 through layers top..stop; returns the vertex reached.  `base`
 // carries the permuted points (and their tensor map) and the degree.
+// With l = e = 1 the loop of warp_search reduces to: N = [(delta(q, c), c)];
+// explore c, compute its neighbours' distances; the lazy check keeps the entries
+// below N's only key (an equal key is c itself); the merge keeps the smallest --
+// so c moves to its nearest neighbour by (dist, id) while that one is nearer,
+// and the search ends when none is.  This form keeps no N, T or bitmap (fewer
+// live registers in the kernels that inline it); results and counters (per
+// layer: 1 + the neighbours of every explored vertex; one iteration per
+// exploration) equal warp_search's at l = e = 1.
 #ifndef GANNS_DESCEND_NOINLINE
 #define GANNS_DESCEND_NOINLINE 0
 #endif
@@ -965,23 +1187,53 @@ struct UpperLayers {
 #else
 #define GANNS_DESCEND_ATTR
 #endif
-template <int NV4, int TPL, bool L2>
+template <int NV4, int TPL, bool L2, bool CPA = false>
 __device__ GANNS_DESCEND_ATTR int32_t descend(const GraphView& base, const UpperLayers& U, int stop,
                            const float* __restrict__ q, WarpSmem& ws,
                            SearchStats* acc = nullptr) {
+  const int lane = threadIdx.x & 31;
+  WarpDist<NV4, L2, CPA> dist;
+  dist.load(base, q, lane);
   int32_t cur = 0;
   for (int j = U.top; j >= stop; --j) {
     GraphView gv = base;
     gv.nbr = U.nbr[j];
     gv.n = U.n[j];
-    SearchStats st;
-    warp_search<NV4, TPL, L2, false>(gv, q, cur, 1, 1, ws, st);
-    if (acc != nullptr) {   // the descent's own counters (bench: its algorithmic bytes)
-      acc->iters += st.iters;
-      acc->comps += st.comps;
+    // N = [(delta(q, cur), cur)]: one distance computation per layer
+    const float dc = __shfl_sync(kFull, dist(gv, lane == 0 ? cur : -1, lane, ws), 0);
+    uint64_t best = mkkey(dc, cur);
+    uint32_t iters = 0, comps = 1;
+    for (;;) {
+      ++iters;
+      const int32_t* row = gv.nbr + size_t(cur) * gv.d_max;
+      int32_t u[TPL];
+#pragma unroll
+      for (int t = 0; t < TPL; ++t) {
+        const int jj = t * 32 + lane;
+        u[t] = jj < gv.d_max ? __ldg(row + jj) : -1;
+      }
+      uint64_t mk = kKeyInf;
+#pragma unroll
+      for (int t = 0; t < TPL; ++t) {
+        const float dd = dist(gv, u[t], lane, ws);
+        const uint64_t kt = u[t] >= 0 ? mkkey(dd, u[t]) : kKeyInf;
+        mk = kt < mk ? kt : mk;
+        comps += __popc(__ballot_sync(kFull, u[t] >= 0));
+      }
+#pragma unroll
+      for (int off = 16; off >= 1; off >>= 1) {
+        const uint64_t o = shfl64(mk, lane ^ off);
+        mk = o < mk ? o : mk;
+      }
+      __syncwarp();   // the stage's reads precede the next gather
+      if (!(mk < best)) break;
+      best = mk;
+      cur = key_id(mk);
     }
-    cur = key_id(unflag(ws.sN[0]));
-    __syncwarp();
+    if (acc != nullptr) {   // the descent's own counters (bench: its algorithmic bytes)
+      acc->iters += iters;
+      acc->comps += comps;
+    }
   }
   return cur;
 }

@@ -66,6 +66,7 @@ inline cudaError_t once_per_device(std::atomic<uint64_t>& done, F&& set) {
 // 1 s of host time (profiles/r02/build_phases_host_gap.log), the pool 0.02 ms.
 cudaError_t pool_alloc(void** p, size_t bytes, cudaStream_t s);
 // GANNS_PROFILE builds: the current device's phase counters (8 x u64), else nullptr
+constexpr int kProfSlots = 16;   // GANNS_PROFILE counters (ganns_dev.cuh, ganns_profile_read_n)
 unsigned long long* prof_buffer();
 void pool_free(void* p, cudaStream_t s);
 

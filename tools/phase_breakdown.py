@@ -29,6 +29,16 @@ def shares(p):
     out["data_structure_ops"] = round(1 - out["distance"] - out["explore"], 4)
     out["cycles_per_iteration"] = round(tot / max(1, p["iterations"]), 1)
     out["iterations_per_search"] = round(p["iterations"] / max(1, p["searches"]), 2)
+    if p.get("gather_rounds") and p.get("spec_build"):
+        out["spec_fill_cycles_per_iteration"] = round(p["gather_issue"] / max(1, p["iterations"]), 1)
+        out["spec_math_cycles_per_iteration"] = round(p["gather_wait"] / max(1, p["iterations"]), 1)
+        out["spec_gathered_ahead_rate"] = round(p["gather_rounds"] / max(1, p["iterations"]), 4)
+    elif p.get("gather_rounds"):
+        r = p["gather_rounds"]
+        out["gather_issue_cycles_per_round"] = round(p["gather_issue"] / r, 1)
+        out["gather_wait_cycles_per_round"] = round(p["gather_wait"] / r, 1)
+        out["gather_rounds_per_iteration"] = round(r / max(1, p["iterations"]), 3)
+        out["spec_hit_rate"] = round(p["spec_hits"] / max(1, p["iterations"]), 4)
     return out
 
 
@@ -41,11 +51,11 @@ if cfg.name != "C4":
     b = g.StagedBuild(Xd, metric=cfg.metric, degree=cfg.degree, l_build=128, l_local=32)
     S, G, dm, dx = b.info()
     b.phase1(0, G)
-    res["build_phase1"] = shares(g.profile_read(reset=True))
+    res["build_phase1"] = shares(dict(g.profile_read(reset=True), spec_build=True))
     for i in range(1, G):
         lo, hi = b.group_rows(i, i + 1)
         b.round_apply(i, *b.round_search(i, lo, hi))
-    res["build_phase2"] = shares(g.profile_read(reset=True))
+    res["build_phase2"] = shares(dict(g.profile_read(reset=True), spec_build=True))
     gr = b.finish()
 idx = BenchIndex(g, cfg, Xd, 128, 32)
 g.profile_read(reset=True)
