@@ -568,7 +568,13 @@ __device__ __forceinline__ void cpasync_fill(const GraphView& g, int32_t u_mine,
 }
 
 // the math over a stage filled by cpasync_fill (its two groups must be this
-// thread's last two commits; any older group is waited for as well)
+// thread's last two commits; any older group is waited for as well).  The stage
+// loads are plain (not lds128_ordered): ptxas may hoist a half's 4 x C loads ahead
+// of its math -- the build searches are latency-bound and have registers to spare
+// (the waits' "memory" clobbers keep every load after its group's wait)
+#ifndef GANNS_CPA_ORDERED
+#define GANNS_CPA_ORDERED 0
+#endif
 template <int S, int C, bool L2, bool FULL>
 __device__ __forceinline__ float cpasync_math(const GraphView& g, const float4 (&qv)[C], int lane,
                                               WarpSmem& ws) {
@@ -589,7 +595,7 @@ __device__ __forceinline__ float cpasync_math(const GraphView& g, const float4 (
     const float4* rp = ws.stage + size_t(gg + S * seg) * g.d4;
     float4 x[C];
 #pragma unroll
-    for (int f = 0; f < C; ++f) x[f] = lds128_ordered(rp + coff[f]);
+    for (int f = 0; f < C; ++f) x[f] = GANNS_CPA_ORDERED ? lds128_ordered(rp + coff[f]) : rp[coff[f]];
     uint64_t acc = 0;
 #pragma unroll
     for (int f = 0; f < C; ++f)

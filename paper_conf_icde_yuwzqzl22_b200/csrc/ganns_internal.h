@@ -164,7 +164,7 @@ struct BuildState {
   int32_t* segoff = nullptr;
   int32_t* touched = nullptr;  // [s * d_min]
   uint64_t* seg = nullptr;     // [s * d_min]
-  int32_t* counters = nullptr; // [2]
+  int32_t* counters = nullptr; // [4]: GatherScatter counters of even / odd rounds
   unsigned long long* stats = nullptr;   // [3] iterations, comps, searches
   CUtensorMap tmap;
   cudaStream_t stream = nullptr;         // the scratch is stream-ordered on this stream
