@@ -26,7 +26,7 @@
 // non-deterministic, and K5 keeps the d_max smallest (dist, id) keys of
 // row ∪ segment, which does not depend on it -- the graph is bit-identical to
 // sorting E by (u, dist, v) (R-C17).
-#include "ganns_dev.cuh"
+#include "search_group.cuh"   // includes ganns_dev.cuh
 #include "../../include/ganns.h"
 #include "ganns_internal.h"
 
@@ -35,6 +35,7 @@
 #endif
 
 #include <algorithm>
+#include <cstdlib>
 #include <cmath>
 #include <new>
 #include <type_traits>
@@ -69,7 +70,22 @@ static cudaError_t launch_pdl(void (*k)(KArgs...), unsigned grid, unsigned block
   return cudaLaunchKernelEx(&cfg, k, static_cast<KArgs>(args)...);
 }
 
-constexpr int kBuildWarps = 1;   // one warp per CTA spreads the latency-bound build searches over all SMs
+constexpr int kBuildWarps = 1;
+// d > 256 (GANNS_BUILD_GROUP): a build search is run by a warp group, as the wide
+// batched search (search_group.cuh): warp 0 runs the loop, all kGroupWarps warps
+// reduce their column slices of each staged row -- one CTA of kGroupWarps warps
+// per search (per group in Phase 1)
+#ifndef GANNS_BUILD_GROUP
+#define GANNS_BUILD_GROUP 1
+#endif
+template <int NV4>
+constexpr bool kBuildGroup = GANNS_BUILD_GROUP != 0 && !uses_tma(NV4);
+template <int NV4>
+constexpr int kBuildThreads = kBuildGroup<NV4> ? kGroupWarps * 32 : kBuildWarps * 32;
+template <int NV4>
+constexpr int kBuildMinBlocks = kBuildGroup<NV4> ? kGroupMinBlocks : 1;
+template <int NV4, bool L2>
+using BuildGroupDist = GroupDist<(NV4 >= 4 ? NV4 / 4 : 1), L2>;   // one warp per CTA spreads the latency-bound build searches over all SMs
 #ifndef GANNS_BUILD_PREDICT
 #define GANNS_BUILD_PREDICT 0
 #endif
@@ -111,16 +127,17 @@ constexpr bool kP1Spec = kBuildSpec<NV4, TPL> && GANNS_BUILD_P1 != 0;
 // Per-warp shared memory of a build search: the search's area, then (cp.async
 // form) T outside the stage
 template <int NV4, int TPL>
-__host__ __device__ constexpr size_t build_warp_bytes(int l, int d4) {
-  return warp_smem_bytes(l, TPL, NV4, d4, kBuildStageRounds) +
+__host__ __device__ constexpr size_t build_warp_bytes(int l, int d4, int wrows) {
+  return warp_smem_bytes(l, TPL, NV4, d4, kBuildStageRounds, wrows) +
          (kBuildCpAsync<NV4> && GANNS_BUILD_T_OUT ? t_bytes(TPL) : 0);
 }
+// wrows: d > 256, rows per TMA round of the build search (BuildDev::wrows_p1/_p2)
 template <int NV4, int TPL>
-__device__ __forceinline__ WarpSmem carve_build_smem(uint8_t* smem, int w, int l, int d4) {
-  uint8_t* base = smem + size_t(w) * build_warp_bytes<NV4, TPL>(l, d4);
-  WarpSmem ws = carve_warp_smem(base, l, TPL, NV4, d4, kBuildStageRounds);
+__device__ __forceinline__ WarpSmem carve_build_smem(uint8_t* smem, int w, int l, int d4, int wrows) {
+  uint8_t* base = smem + size_t(w) * build_warp_bytes<NV4, TPL>(l, d4, wrows);
+  WarpSmem ws = carve_warp_smem(base, l, TPL, NV4, d4, kBuildStageRounds, wrows);
   if constexpr (kBuildCpAsync<NV4> && GANNS_BUILD_T_OUT) {
-    ws.sT = reinterpret_cast<uint64_t*>(base + warp_smem_bytes(l, TPL, NV4, d4, kBuildStageRounds));
+    ws.sT = reinterpret_cast<uint64_t*>(base + warp_smem_bytes(l, TPL, NV4, d4, kBuildStageRounds, wrows));
   }
   return ws;
 }
@@ -186,6 +203,7 @@ struct BuildDev {
   float* gpd;
   int d_min, l_build, e_build;
   int l_local, e_local;   // Phase-1 searches on the local graphs (<= l_build)
+  int wrows_p1, wrows_p2;   // d > 256: rows per TMA round in Phase 1 / Phase 2
   unsigned long long* stats;   // [3] iterations, comps, searches
 };
 
@@ -200,17 +218,30 @@ __device__ __forceinline__ void add_stats(unsigned long long* st, const SearchSt
 // ------------------------------------------------------------------ K2
 // Phase 1: local graph construction (Alg. 2 lines 2-8).
 template <int NV4, int TPL, bool L2>
-__global__ void __launch_bounds__(kBuildWarps * 32)
+__global__ void __launch_bounds__(kBuildThreads<NV4>, kBuildMinBlocks<NV4>)
 phase1_kernel(BuildDev B, int64_t group_size, int64_t g0, int64_t g1,
               const __grid_constant__ CUtensorMap tmap) {
   B.g.tmap = &tmap;
   extern __shared__ __align__(128) uint8_t smem[];
+  constexpr bool GROUP = kBuildGroup<NV4>;
   const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int64_t gi = g0 + int64_t(blockIdx.x) * kBuildWarps + w;   // groups [g0, g1)
+  const int64_t gi = g0 + int64_t(blockIdx.x) * kBuildWarps + (GROUP ? 0 : w);   // groups [g0, g1)
   if (gi >= g1) return;
-  WarpSmem ws = carve_build_smem<NV4, TPL>(smem, w, B.l_build, B.g.d4);
-  if (lane == 0) mbar_init(ws.mbar, 1);
-  __syncwarp();
+  WarpSmem ws = carve_build_smem<NV4, TPL>(smem, GROUP ? 0 : w, B.l_build, B.g.d4, B.wrows_p1);
+  BuildGroupDist<NV4, L2> gdist;
+  if constexpr (GROUP) {
+    gdist.gs = carve_group(smem + build_warp_bytes<NV4, TPL>(B.l_build, B.g.d4, B.wrows_p1));
+    gdist.kc = 0;
+    if (threadIdx.x == 0) mbar_init(ws.mbar, 1);
+    __syncthreads();
+    if (w != 0) {
+      group_helper_loop<(NV4 >= 4 ? NV4 / 4 : 1), L2>(B.g, B.g.X, gdist.gs, ws, w, lane);
+      return;
+    }
+  } else {
+    if (lane == 0) mbar_init(ws.mbar, 1);
+    __syncwarp();
+  }
   uint64_t* sN = ws.sN;
   const int64_t lo = gi * group_size;
   const int64_t hi = lo + group_size < B.g.n ? lo + group_size : B.g.n;
@@ -218,8 +249,15 @@ phase1_kernel(BuildDev B, int64_t group_size, int64_t g0, int64_t g1,
   for (int64_t v = lo + 1; v < hi; ++v) {
     // Step 1 (line 5): v.N, v.N' := Search(G_i, v, d_min), entry = group's first vertex
     SearchStats st;
-    const int cnt = warp_search<NV4, TPL, L2, true, kBuildPredict, kP1Spec<NV4, TPL>, kP1CpAsync<NV4>>(
-        B.g, B.g.X + size_t(v) * d, int32_t(lo), B.l_local, B.e_local, ws, st);
+    int cnt;
+    if constexpr (GROUP) {
+      group_new_query(gdist, B.g, B.g.X, v, lane);
+      cnt = warp_search_with<BuildGroupDist<NV4, L2>, TPL, true>(B.g, gdist, int32_t(lo), B.l_local,
+                                                                 B.e_local, ws, st);
+    } else {
+      cnt = warp_search<NV4, TPL, L2, true, kBuildPredict, kP1Spec<NV4, TPL>, kP1CpAsync<NV4>>(
+          B.g, B.g.X + size_t(v) * d, int32_t(lo), B.l_local, B.e_local, ws, st);
+    }
     add_stats(B.stats, st, lane);
     const int m = cnt < B.d_min ? cnt : B.d_min;
     for (int j = lane; j < m; j += 32) {
@@ -252,6 +290,7 @@ phase1_kernel(BuildDev B, int64_t group_size, int64_t g0, int64_t g1,
       __syncwarp();
     }
   }
+  if constexpr (GROUP) gdist.post(kCmdExit, lane);
 }
 
 // ------------------------------------------------------------------ K3
@@ -264,7 +303,7 @@ phase1_kernel(BuildDev B, int64_t group_size, int64_t g0, int64_t g1,
 // HNSW: the instance that enters through the descent of the upper layers (the
 // plain NSW build's instance carries no descent code)
 template <int NV4, int TPL, bool L2, bool HNSW>
-__global__ void __launch_bounds__(kBuildWarps * 32)
+__global__ void __launch_bounds__(kBuildThreads<NV4>, kBuildMinBlocks<NV4>)
 round_search_kernel(BuildDev B, int64_t lo, int64_t v0, int64_t v1, int32_t* __restrict__ Eu,
                     float* __restrict__ Ed, int32_t* __restrict__ indeg,
                     int32_t* __restrict__ touched, int32_t* __restrict__ counters,
@@ -273,12 +312,29 @@ round_search_kernel(BuildDev B, int64_t lo, int64_t v0, int64_t v1, int32_t* __r
   pdl_wait();   // G_0 as the previous round's K5 left it
   B.g.tmap = &tmap;
   extern __shared__ __align__(128) uint8_t smem[];
+  // the HNSW instance keeps the one-warp form (its descent is the leader's alone)
+  constexpr bool GROUP = kBuildGroup<NV4> && !HNSW;
   const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int64_t v = v0 + int64_t(blockIdx.x) * kBuildWarps + w;
+  const int64_t v = v0 + int64_t(blockIdx.x) * kBuildWarps + (kBuildGroup<NV4> ? 0 : w);
   if (v >= v1) return;
-  WarpSmem ws = carve_build_smem<NV4, TPL>(smem, w, B.l_build, B.g.d4);
-  if (lane == 0) mbar_init(ws.mbar, 1);
-  __syncwarp();
+  if constexpr (kBuildGroup<NV4> && HNSW)
+    if (w != 0) return;
+  WarpSmem ws = carve_build_smem<NV4, TPL>(smem, kBuildGroup<NV4> ? 0 : w, B.l_build, B.g.d4,
+                                           B.wrows_p2);
+  BuildGroupDist<NV4, L2> gdist;
+  if constexpr (GROUP) {
+    gdist.gs = carve_group(smem + build_warp_bytes<NV4, TPL>(B.l_build, B.g.d4, B.wrows_p2));
+    gdist.kc = 0;
+    if (threadIdx.x == 0) mbar_init(ws.mbar, 1);
+    __syncthreads();
+    if (w != 0) {
+      group_helper_loop<(NV4 >= 4 ? NV4 / 4 : 1), L2>(B.g, B.g.X, gdist.gs, ws, w, lane);
+      return;
+    }
+  } else {
+    if (lane == 0) mbar_init(ws.mbar, 1);
+    __syncwarp();
+  }
   uint64_t* sN = ws.sN;
   uint64_t* sT = ws.sT;
   const int d = B.g.d4 * 4;
@@ -294,8 +350,16 @@ round_search_kernel(BuildDev B, int64_t lo, int64_t v0, int64_t v1, int32_t* __r
     }
   }
   SearchStats st;
-  const int cnt = warp_search<NV4, TPL, L2, false, kBuildPredict, kBuildSpec<NV4, TPL>, kBuildCpAsync<NV4>>(
-      B.g, B.g.X + size_t(v) * d, entry, B.l_build, B.e_build, ws, st);
+  int cnt;
+  if constexpr (GROUP) {
+    group_new_query(gdist, B.g, B.g.X, v, lane);
+    cnt = warp_search_with<BuildGroupDist<NV4, L2>, TPL, false>(B.g, gdist, entry, B.l_build,
+                                                                B.e_build, ws, st);
+    gdist.post(kCmdExit, lane);
+  } else {
+    cnt = warp_search<NV4, TPL, L2, false, kBuildPredict, kBuildSpec<NV4, TPL>, kBuildCpAsync<NV4>>(
+        B.g, B.g.X + size_t(v) * d, entry, B.l_build, B.e_build, ws, st);
+  }
   add_stats(B.stats, st, lane);
   const int dm = B.d_min;
   const int cs = cnt < dm ? cnt : dm;
@@ -504,7 +568,7 @@ static __global__ void fill_rows_kernel(int32_t* ids, float* dists, int64_t coun
 struct BuildDevState {
   BuildDev B;
   UpperLayers U;
-  size_t smem;
+  size_t smem_p1, smem_p2;
 };
 
 template <int NV4, int TPL, bool L2>
@@ -513,7 +577,7 @@ static int phase1_t(BuildState& st, int64_t g0, int64_t g1, cudaStream_t s) {
   if (g1 <= g0) return 0;
   // all local graphs of [g0, g1) in parallel, one warp per group (lines 2-8)
   phase1_kernel<NV4, TPL, L2><<<unsigned((g1 - g0 + kBuildWarps - 1) / kBuildWarps),
-                                kBuildWarps * 32, ds->smem, s>>>(ds->B, st.S, g0, g1, st.tmap);
+                                kBuildThreads<NV4>, ds->smem_p1, s>>>(ds->B, st.S, g0, g1, st.tmap);
   count_launch();
   GANNS_TRY(cudaGetLastError());
   return 0;
@@ -532,11 +596,11 @@ static int round_search_t(BuildState& st, int64_t i, int64_t v0, int64_t v1, int
   // K5, or at begin for rounds 1 and 2)
   const unsigned grid = unsigned((v1 - v0 + kBuildWarps - 1) / kBuildWarps);
   if (ds->U.top > st.a.layer)
-    GANNS_TRY(launch_pdl(round_search_kernel<NV4, TPL, L2, true>, grid, kBuildWarps * 32, ds->smem,
+    GANNS_TRY(launch_pdl(round_search_kernel<NV4, TPL, L2, true>, grid, kBuildThreads<NV4>, ds->smem_p2,
                          s, ds->B, lo, v0, v1, st.Eu, st.Ed, st.indeg, st.touched,
                          round_counters(st, i), f_ids, f_dists, st.tmap, ds->U, st.a.layer));
   else
-    GANNS_TRY(launch_pdl(round_search_kernel<NV4, TPL, L2, false>, grid, kBuildWarps * 32, ds->smem,
+    GANNS_TRY(launch_pdl(round_search_kernel<NV4, TPL, L2, false>, grid, kBuildThreads<NV4>, ds->smem_p2,
                          s, ds->B, lo, v0, v1, st.Eu, st.Ed, st.indeg, st.touched,
                          round_counters(st, i), f_ids, f_dists, st.tmap, ds->U, st.a.layer));
   count_launch();
@@ -625,8 +689,22 @@ static int begin_t(BuildState& st, cudaStream_t s) {
   B.l_local = a.l_local > 0 ? a.l_local : a.l_build;
   B.e_local = a.e_local > 0 ? a.e_local : a.e_build;
   B.stats = st.stats;
-  ds->smem = size_t(kBuildWarps) * build_warp_bytes<NV4, TPL>(a.l_build, a.d / 4);
-  if (ds->smem > 227 * 1024) return fail(GANNS_ENOTSUP, "build: shared memory per CTA exceeds 227 KB");
+  // d > 256: rows per TMA round (1-D bulk copies); GANNS_BUILD_WROWS overrides the
+  // default 8.  Fitting a round's searches into one wave of resident warps with
+  // fewer rows per round was measured slower on C3 (3.12 s at R = 8 in 1.5 waves,
+  // 3.17 s at R = 5, 3.31 s at R = 4): the second wave runs in the first one's
+  // tail (a round lasts as long as its slowest search)
+  static const int forced_wrows = [] {
+    const char* e = std::getenv("GANNS_BUILD_WROWS");
+    const int r = e ? std::atoi(e) : 0;
+    return r >= 1 && r <= kWideStageRows ? r : kWideStageRows;
+  }();
+  B.wrows_p1 = B.wrows_p2 = forced_wrows;
+  const size_t garea = kBuildGroup<NV4> ? group_area_bytes() : 0;
+  ds->smem_p1 = size_t(kBuildWarps) * build_warp_bytes<NV4, TPL>(a.l_build, a.d / 4, B.wrows_p1) + garea;
+  ds->smem_p2 = size_t(kBuildWarps) * build_warp_bytes<NV4, TPL>(a.l_build, a.d / 4, B.wrows_p2) + garea;
+  if (std::max(ds->smem_p1, ds->smem_p2) > 227 * 1024)
+    return fail(GANNS_ENOTSUP, "build: shared memory per CTA exceeds 227 KB");
   ds->U.top = a.upper.top;
   for (int j = 0; j < kMaxLayers; ++j) {
     ds->U.nbr[j] = a.upper.nbr[j];

@@ -175,6 +175,50 @@ struct GroupDist {
   }
 };
 
+// Helper warps (w != 0): execute the leader's commands until it posts kCmdExit.
+// A new query's row is Q[*gs.sQ] (the search's queries, or the build's points).
+template <int CG, bool L2>
+__device__ __forceinline__ void group_helper_loop(const GraphView& g, const float* __restrict__ Q,
+                                                  const GroupShared& gs, WarpSmem& ws, int w,
+                                                  int lane) {
+  float4 qv[CG];
+  int kc = 0;
+  for (;;) {
+    group_bar(1);
+    const int cmd = gs.sCmd[kc & 1];
+    ++kc;
+    if (cmd == kCmdExit) return;
+    if (cmd == kCmdNewQuery) {
+      const float s = group_load_query<CG>(g, Q + size_t(*gs.sQ) * (g.d4 * 4), w, lane, qv);
+      if (lane == 0) gs.sNorm[w] = s;
+      group_bar(2);
+      continue;
+    }
+    group_rounds<CG, L2, false>(g, qv, gs.sU[lane], lane, w, ws, gs.sPart);
+  }
+}
+
+// Leader: start the group's search of row q of Q (every warp loads its query slice;
+// cosine needs the full |q|).
+template <int CG, bool L2>
+__device__ __forceinline__ void group_new_query(GroupDist<CG, L2>& dist, const GraphView& g,
+                                                const float* __restrict__ Q, int64_t q, int lane) {
+  if (lane == 0) *dist.gs.sQ = q;
+  dist.post(kCmdNewQuery, lane);
+  const float s0 = group_load_query<CG>(g, Q + size_t(q) * (g.d4 * 4), 0, lane, dist.qv);
+  if (lane == 0) dist.gs.sNorm[0] = s0;
+  group_bar(2);
+  dist.cbase = 0.f;
+  dist.qinv = 1.f;
+  if (!L2 && g.metric == 2) {
+    float s = 0.f;
+#pragma unroll
+    for (int i = 0; i < kGroupWarps; ++i) s += dist.gs.sNorm[i];
+    dist.cbase = 1.f;
+    dist.qinv = 1.f / sqrtf(s);
+  }
+}
+
 template <int CG, int TPL, bool L2>
 __global__ void __launch_bounds__(kGroupWarps * 32, kGroupMinBlocks)
 search_group_kernel(GraphView g, const float* __restrict__ Q, int64_t nq, int k, int l, int e,
@@ -188,24 +232,9 @@ search_group_kernel(GraphView g, const float* __restrict__ Q, int64_t nq, int k,
   GroupShared gs = carve_group(smem + wsb);
   if (threadIdx.x == 0) mbar_init(ws.mbar, 1);
   __syncthreads();
-  const bool cosine = !L2 && g.metric == 2;
   if (w != 0) {
-    // helper warps: execute the leader's commands until it posts kCmdExit
-    float4 qv[CG];
-    int kc = 0;
-    for (;;) {
-      group_bar(1);
-      const int cmd = gs.sCmd[kc & 1];
-      ++kc;
-      if (cmd == kCmdExit) return;
-      if (cmd == kCmdNewQuery) {
-        const float s = group_load_query<CG>(g, Q + size_t(*gs.sQ) * (g.d4 * 4), w, lane, qv);
-        if (lane == 0) gs.sNorm[w] = s;
-        group_bar(2);
-        continue;
-      }
-      group_rounds<CG, L2, false>(g, qv, gs.sU[lane], lane, w, ws, gs.sPart);
-    }
+    group_helper_loop<CG, L2>(g, Q, gs, ws, w, lane);
+    return;
   }
   GroupDist<CG, L2> dist;
   dist.gs = gs;
@@ -219,20 +248,7 @@ search_group_kernel(GraphView g, const float* __restrict__ Q, int64_t nq, int k,
       dist.post(kCmdExit, lane);
       break;
     }
-    if (lane == 0) *gs.sQ = q;
-    dist.post(kCmdNewQuery, lane);
-    const float s0 = group_load_query<CG>(g, Q + size_t(q) * (g.d4 * 4), 0, lane, dist.qv);
-    if (lane == 0) gs.sNorm[0] = s0;
-    group_bar(2);
-    dist.cbase = 0.f;
-    dist.qinv = 1.f;
-    if (cosine) {
-      float s = 0.f;
-#pragma unroll
-      for (int i = 0; i < kGroupWarps; ++i) s += gs.sNorm[i];
-      dist.cbase = 1.f;
-      dist.qinv = 1.f / sqrtf(s);
-    }
+    group_new_query<CG, L2>(dist, g, Q, q, lane);
     SearchStats st;
     const int32_t ent = entries != nullptr ? entries[q] : entry;   // HNSW: per-query entry
     const int cnt = warp_search_with<GroupDist<CG, L2>, TPL, false>(g, dist, ent, l, e, ws, st);

@@ -101,3 +101,18 @@ def test_build_parity_l_local(l_local):
     ref, _, _ = oracle.alg2(X, 8, 16, 256, l_build=64, l_local=l_local)
     _, adj = gpu_build(X, 16, l_build=64, group_size=256, l_local=l_local)
     assert (adj == ref).all()
+
+
+@pytest.mark.parametrize("d,metric,s", [(384, "l2", 300), (960, "l2", 256), (960, "ip", 500)])
+def test_build_parity_wide_rows_group(d, metric, s):
+    """d > 256: the build searches run on a warp group (warp 0 the GANNS loop, all
+    four warps the column slices of the bulk distance, search_group.cuh) -- Phase 1
+    and Phase 2 equal the oracle's Algorithm 2 (adjacency and counters)."""
+    cfg = syn.with_size(syn.CONFIGS["C3"], n=2500)
+    X = np.ascontiguousarray(syn.points(cfg)[:, :d])
+    if metric == "ip":
+        X = X - 8.0   # signed integer grid: exact inner products
+    ref, _, st = oracle.alg2(X, 16, 32, s, l_build=64, l_local=32, metric=metric)
+    graph, adj = gpu_build(X, 32, l_build=64, l_local=32, group_size=s, metric=metric)
+    assert (adj == ref).all(), np.argwhere(adj != ref)[:5]
+    assert tuple(graph.build_stats[:3]) == tuple(int(x) for x in st)
