@@ -513,60 +513,89 @@ __device__ __forceinline__ float tma_dot(const GraphView& g, const float4 (&qv)[
 }
 
 // One-round segment form with the stage filled by per-lane async copies
-// (cp.async.cg, SASS LDGSTS: 16 B per lane, one warp instruction per 512 B of a
-// row, L2 only) instead of TMA -- the form of the build searches (ws.cpasync).
-// The row of lane L goes to slot L as in tma_dot's one-round layout, so the math
-// is the same.  Rows are copied in pass order in two commit groups: the first
-// half of the passes starts its math while the second half's rows still arrive.
-// No mbarrier and no uniform-register issue loop (a tile::gather4 per 4 rows
-// costs one ELECT / R2UR waterfall iteration per issuing lane), and no proxy
-// fence: cp.async writes are generic-proxy writes.
+// (cp.async.cg, SASS LDGSTS: 16 B per lane, 512 B per warp instruction, L2 only)
+// instead of TMA -- the form of the build searches (CPA).  The row of lane L goes
+// to slot L as in tma_dot's one-round layout, so the math is the same.  Rows are
+// copied in pass order in two commit groups: the first half of the passes starts
+// its math while the second half's rows still arrive.  No mbarrier and no
+// uniform-register issue loop (a tile::gather4 per 4 rows costs one ELECT / R2UR
+// waterfall iteration per issuing lane), and no proxy fence: cp.async writes are
+// generic-proxy writes.
 __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+// 4 x 16 B at byte offsets 0, 128, 256, 384 of src -> dst, where u >= 0 (one
+// predicate, no branch)
+__device__ __forceinline__ void cp_async_4x128(uint32_t dst, const void* src, int32_t u) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\tsetp.ge.s32 p, %2, 0;\n\t"
+      "@p cp.async.cg.shared.global [%0], [%1], 16;\n\t"
+      "@p cp.async.cg.shared.global [%0+128], [%1+128], 16;\n\t"
+      "@p cp.async.cg.shared.global [%0+256], [%1+256], 16;\n\t"
+      "@p cp.async.cg.shared.global [%0+384], [%1+384], 16;\n\t}" ::"r"(dst),
+      "l"(src), "r"(u)
+      : "memory");
+}
 template <int N>
 __device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
-// 16 B of row u (u >= 0; else nothing) at byte offset `src` of the rows' base
-// (the lane's chunk) -> shared address dst: one predicate, one address, one copy
-__device__ __forceinline__ void cp_async_row16(uint32_t dst, const void* src, int32_t u,
-                                               uint32_t rowbytes) {
+// 4 x 16 B at byte offsets 0, 128, 256, 384 of src -> dst, copy i where u >= 0 and
+// bit i of mask (the row's tail chunks of a d that is not a multiple of 32 floats)
+__device__ __forceinline__ void cp_async_4x128_m(uint32_t dst, const void* src, int32_t u,
+                                                 uint32_t mask) {
   asm volatile(
-      "{\n\t.reg .pred p;\n\t.reg .u64 a;\n\tsetp.ge.s32 p, %2, 0;\n\t"
-      "mad.wide.u32 a, %2, %3, %1;\n\t@p cp.async.cg.shared.global [%0], [a], 16;\n\t}" ::"r"(dst),
-      "l"(src), "r"(u), "r"(rowbytes)
+      "{\n\t.reg .pred p, q0, q1, q2, q3;\n\t.reg .b32 t;\n\tsetp.ge.s32 p, %2, 0;\n\t"
+      "and.b32 t, %3, 1;\n\tsetp.ne.and.b32 q0, t, 0, p;\n\t"
+      "and.b32 t, %3, 2;\n\tsetp.ne.and.b32 q1, t, 0, p;\n\t"
+      "and.b32 t, %3, 4;\n\tsetp.ne.and.b32 q2, t, 0, p;\n\t"
+      "and.b32 t, %3, 8;\n\tsetp.ne.and.b32 q3, t, 0, p;\n\t"
+      "@q0 cp.async.cg.shared.global [%0], [%1], 16;\n\t"
+      "@q1 cp.async.cg.shared.global [%0+128], [%1+128], 16;\n\t"
+      "@q2 cp.async.cg.shared.global [%0+256], [%1+256], 16;\n\t"
+      "@q3 cp.async.cg.shared.global [%0+384], [%1+384], 16;\n\t}" ::"r"(dst),
+      "l"(src), "r"(u), "r"(mask)
       : "memory");
 }
 
-// issue the copies of the <= 32 rows (u_mine per lane, -1 = none) into the stage:
-// one warp instruction per 512 B of a row (lane c copies 16-B chunk c, and c + 32
-// for d > 128), straight-line and predicated -- per row a shuffle of its id, a
-// predicate, an address and the copy (a branchy per-row loop cost ~18
-// instructions per row and instruction-cache misses); two commit groups (the rows
-// of passes [0, S/2), then [S/2, S)).  FULL: d = 4 * S * C, the row size is a
-// compile-time constant (the stage offsets become immediates).
-template <int S, bool FULL>
-__device__ __forceinline__ void cpasync_fill(const GraphView& g, int32_t u_mine, int lane,
-                                             const WarpSmem& ws) {
-  constexpr int NSEG = 32 / S;
-  constexpr int CH = S / 8;   // 16-B chunks per lane per row: d <= 128 -> 1, d <= 256 -> 2
-  const uint32_t rowbytes = FULL ? uint32_t(S) * 64u : uint32_t(g.d4) * 16u;
-  const uint32_t sbase = smem_u32(ws.stage) + uint32_t(lane) * 16u;
-  const char* xb = reinterpret_cast<const char*>(g.X) + lane * 16;
-  bool in[CH];
+// cpasync_fill_quad: each copy instruction moves 4 rows x 128 B -- lanes 8r..8r+7
+// copy 16-B chunks c = lane % 8 + 8 j of row 4k + r -- so a lane needs the ids of 8
+// rows (8 shuffles, 8 addresses, one predicate per 4 copies) for its 32 (d = 128)
+// or 64 (d = 256) copies: ~90 instructions per exploration at d = 128, against 160
+// with one row per instruction (a shuffle, predicate and address per row; Phase 1
+// 0.0955 -> 0.0929 s) and ~580 for a first version with a per-row copy loop
+// (instruction-cache misses; 3x slower builds).
+// Other d (d % 4 == 0, a row of d4 16-B chunks): the same layout with the row size
+// at run time and the chunks >= d4 masked off (FULL = false).
+template <int S, bool FULL = true>
+__device__ __forceinline__ void cpasync_fill_quad(const GraphView& g, int32_t u_mine, int lane,
+                                                  const WarpSmem& ws) {
+  const uint32_t rowbytes = FULL ? uint32_t(S) * 64u : uint32_t(g.d4) * 16u;   // FULL: d4 = S * C
+  constexpr int NJ = S / 2;                          // 16-B chunks per lane per row (max)
+  const int r = lane >> 3, c0 = lane & 7;
+  uint32_t cmask[NJ / 4];   // chunks c0 + 8 j < d4, 4 per copy block
 #pragma unroll
-  for (int j = 0; j < CH; ++j) in[j] = FULL || lane + 32 * j < g.d4;
+  for (int b = 0; b < NJ / 4; ++b) {
+    cmask[b] = 0;
 #pragma unroll
-  for (int gg = 0; gg < S; ++gg) {
-#pragma unroll
-    for (int s = 0; s < NSEG; ++s) {
-      const int L = gg + S * s;
-      const int32_t u = __shfl_sync(kFull, u_mine, L);
-#pragma unroll
-      for (int j = 0; j < CH; ++j)
-        cp_async_row16(sbase + uint32_t(L) * rowbytes + 512u * j, xb + 512 * j, in[j] ? u : -1,
-                       rowbytes);
-    }
-    if (gg == S / 2 - 1) cp_async_commit();
+    for (int i = 0; i < 4; ++i) cmask[b] |= (FULL || c0 + 8 * (4 * b + i) < g.d4) ? (1u << i) : 0u;
   }
-  cp_async_commit();
+  const uint32_t sbase = smem_u32(ws.stage) + uint32_t(r) * rowbytes + uint32_t(c0) * 16u;
+  const char* xb = reinterpret_cast<const char*>(g.X) + c0 * 16;
+#pragma unroll
+  for (int h = 0; h < 2; ++h) {
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+      // row quad k (rows 4k..4k+3) belongs to the first half of the passes iff its
+      // rows' pass index (row % S) is < S / 2
+      if (((4 * k) % S < S / 2) != (h == 0)) continue;
+      const int32_t u = __shfl_sync(kFull, u_mine, 4 * k + r);
+      const uint32_t dst = sbase + uint32_t(4 * k) * rowbytes;
+      const char* src = xb + uint64_t(uint32_t(u >= 0 ? u : 0)) * rowbytes;
+#pragma unroll
+      for (int j = 0; j < NJ; j += 4) {
+        if constexpr (FULL) cp_async_4x128(dst + 128u * j, src + 128 * j, u);
+        else cp_async_4x128_m(dst + 128u * j, src + 128 * j, u, cmask[j / 4]);
+      }
+    }
+    cp_async_commit();
+  }
 }
 
 // the math over a stage filled by cpasync_fill (its two groups must be this
@@ -698,10 +727,10 @@ __device__ __forceinline__ float group_distances(const GraphView& g,
   if constexpr (S < 32) {
     if constexpr (CPA) {
       if (full) {
-        cpasync_fill<S, true>(g, u_mine, lane, ws);
+        cpasync_fill_quad<S>(g, u_mine, lane, ws);
         dot = cpasync_math<S, C, L2, true>(g, qv, lane, ws);
       } else {
-        cpasync_fill<S, false>(g, u_mine, lane, ws);
+        cpasync_fill_quad<S, false>(g, u_mine, lane, ws);
         dot = cpasync_math<S, C, L2, false>(g, qv, lane, ws);
       }
     } else if (ws.rounds == 1)
@@ -768,8 +797,8 @@ struct WarpDist {
   // issued by fill() -- possibly one iteration early -- and reduced by math()
   __device__ __forceinline__ void fill(const GraphView& g, int32_t u_mine, int lane, WarpSmem& ws) {
     if constexpr (uses_tma(NV4)) {
-      if (g.d4 == S * C) cpasync_fill<S, true>(g, u_mine, lane, ws);
-      else cpasync_fill<S, false>(g, u_mine, lane, ws);
+      if (g.d4 == S * C) cpasync_fill_quad<S>(g, u_mine, lane, ws);
+      else cpasync_fill_quad<S, false>(g, u_mine, lane, ws);
     }
   }
   template <int PEND = 0>
