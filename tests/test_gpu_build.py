@@ -116,3 +116,28 @@ def test_build_parity_wide_rows_group(d, metric, s):
     graph, adj = gpu_build(X, 32, l_build=64, l_local=32, group_size=s, metric=metric)
     assert (adj == ref).all(), np.argwhere(adj != ref)[:5]
     assert tuple(graph.build_stats[:3]) == tuple(int(x) for x in st)
+
+
+@pytest.mark.parametrize("n,d,degree,l_build,l_local,s,metric", [
+    (1800, 24, 16, 48, 16, 200, "l2"),     # d4 = 6: masked tail chunks (S = 8)
+    (1800, 100, 32, 64, 32, 300, "l2"),    # d4 = 25
+    (1500, 200, 32, 96, 32, 256, "ip"),    # d4 = 50 (S = 16, masked), C4's row width
+    (1500, 256, 32, 64, 24, 250, "l2"),    # d4 = 64 (S = 16, full)
+    (1200, 128, 24, 40, 40, 128, "l2"),    # d_max 24 < 32: partial adjacency rows
+    (1600, 128, 32, 128, 32, 1600, "l2"),  # one group: Phase 1 only
+    (2000, 128, 32, 32, 16, 64, "l2"),     # many small rounds
+])
+def test_build_parity_cpasync_speculation_shapes(n, d, degree, l_build, l_local, s, metric):
+    """The build searches' cp.async four-row fill (full and masked rows), the
+    speculative gather of the next candidate, and programmatic dependent launch
+    across many rounds: adjacency and counters equal the oracle's Algorithm 2."""
+    rng = np.random.default_rng(n + d)
+    X = rng.integers(0, 16, size=(n, d)).astype(np.float32)
+    if metric == "ip":
+        X = X - 8.0
+    ref, _, st = oracle.alg2(X, degree // 2, degree, s, l_build=l_build, l_local=l_local,
+                             metric=metric, threads=4)
+    graph, adj = gpu_build(X, degree, l_build=l_build, l_local=l_local, group_size=s,
+                           metric=metric)
+    assert (adj == ref).all(), np.argwhere(adj != ref)[:5]
+    assert tuple(graph.build_stats[:3]) == tuple(int(x) for x in st)
