@@ -123,16 +123,6 @@ template <int NV4>
 constexpr bool kP1CpAsync = kBuildCpAsync<NV4> && GANNS_BUILD_P1 != 0;
 template <int NV4, int TPL>
 constexpr bool kP1Spec = kBuildSpec<NV4, TPL> && GANNS_BUILD_P1 != 0;
-// GANNS_BUILD_P1_DBL: the Phase-1 searches (one warp per group, ~4.4 per SM: shared
-// memory to spare) keep a second stage, so the speculative gather is issued before
-// the current math and a miss never waits for a stale speculation (warp_search_with,
-// DBL).  Off: measured Phase 1 0.0953 -> 0.1012 s with it (the speculative fill's
-// issue then sits before the math on every iteration)
-#ifndef GANNS_BUILD_P1_DBL
-#define GANNS_BUILD_P1_DBL 0
-#endif
-template <int NV4, int TPL>
-constexpr bool kP1Dbl = kP1Spec<NV4, TPL> && GANNS_BUILD_P1_DBL != 0;
 #ifndef GANNS_BUILD_T_OUT
 #define GANNS_BUILD_T_OUT 1
 #endif
@@ -241,8 +231,6 @@ phase1_kernel(BuildDev B, int64_t group_size, int64_t g0, int64_t g1,
   const int64_t gi = g0 + int64_t(blockIdx.x) * kBuildWarps + (GROUP ? 0 : w);   // groups [g0, g1)
   if (gi >= g1) return;
   WarpSmem ws = carve_build_smem<NV4, TPL>(smem, GROUP ? 0 : w, B.l_build, B.g.d4, B.wrows_p1);
-  if constexpr (kP1Dbl<NV4, TPL>)   // kBuildWarps == 1: the second stage follows the warp's area
-    ws.stage2 = reinterpret_cast<float4*>(smem + build_warp_bytes<NV4, TPL>(B.l_build, B.g.d4, B.wrows_p1));
   BuildGroupDist<NV4, L2> gdist;
   if constexpr (GROUP) {
     gdist.gs = carve_group(smem + build_warp_bytes<NV4, TPL>(B.l_build, B.g.d4, B.wrows_p1));
@@ -270,9 +258,8 @@ phase1_kernel(BuildDev B, int64_t group_size, int64_t g0, int64_t g1,
       cnt = warp_search_with<BuildGroupDist<NV4, L2>, TPL, true>(B.g, gdist, int32_t(lo), B.l_local,
                                                                  B.e_local, ws, st);
     } else {
-      cnt = warp_search<NV4, TPL, L2, true, kBuildPredict, kP1Spec<NV4, TPL>, kP1CpAsync<NV4>,
-                        kP1Dbl<NV4, TPL>>(B.g, B.g.X + size_t(v) * d, int32_t(lo), B.l_local,
-                                          B.e_local, ws, st);
+      cnt = warp_search<NV4, TPL, L2, true, kBuildPredict, kP1Spec<NV4, TPL>, kP1CpAsync<NV4>>(
+          B.g, B.g.X + size_t(v) * d, int32_t(lo), B.l_local, B.e_local, ws, st);
     }
     add_stats(B.stats, st, lane);
     const int m = cnt < B.d_min ? cnt : B.d_min;
@@ -717,8 +704,7 @@ static int begin_t(BuildState& st, cudaStream_t s) {
   }();
   B.wrows_p1 = B.wrows_p2 = forced_wrows;
   const size_t garea = kBuildGroup<NV4> ? group_area_bytes() : 0;
-  ds->smem_p1 = size_t(kBuildWarps) * build_warp_bytes<NV4, TPL>(a.l_build, a.d / 4, B.wrows_p1) + garea +
-                (kP1Dbl<NV4, TPL> ? stage_bytes(NV4, a.d / 4, kBuildStageRounds) : 0);
+  ds->smem_p1 = size_t(kBuildWarps) * build_warp_bytes<NV4, TPL>(a.l_build, a.d / 4, B.wrows_p1) + garea;
   ds->smem_p2 = size_t(kBuildWarps) * build_warp_bytes<NV4, TPL>(a.l_build, a.d / 4, B.wrows_p2) + garea;
   if (std::max(ds->smem_p1, ds->smem_p2) > 227 * 1024)
     return fail(GANNS_ENOTSUP, "build: shared memory per CTA exceeds 227 KB");

@@ -254,8 +254,6 @@ struct WarpSmem {
   float4* pair_stage;
   volatile int* pair_flag;
   int pair_bar;   // named barrier of the pair (64 threads): leaver arrives, taker syncs
-  // SPEC with a second stage (DBL, the Phase-1 build searches: few warps per SM)
-  float4* stage2 = nullptr;
 #if GANNS_PROFILE
   unsigned long long p_issue = 0, p_wait = 0, p_rounds = 0;   // lane 0's gather timers
 #endif
@@ -606,9 +604,7 @@ __device__ __forceinline__ void cpasync_fill_quad(const GraphView& g, int32_t u_
 #ifndef GANNS_CPA_ORDERED
 #define GANNS_CPA_ORDERED 0
 #endif
-// PEND: groups committed after this stage's two (a speculative fill of the other
-// stage, DBL) that the waits leave in flight
-template <int S, int C, bool L2, bool FULL, int PEND = 0>
+template <int S, int C, bool L2, bool FULL>
 __device__ __forceinline__ float cpasync_math(const GraphView& g, const float4 (&qv)[C], int lane,
                                               WarpSmem& ws) {
   const int sl = lane & (S - 1), seg = lane / S;
@@ -619,10 +615,10 @@ __device__ __forceinline__ float cpasync_math(const GraphView& g, const float4 (
 #pragma unroll
   for (int gg = 0; gg < S; ++gg) {
     if (gg == 0) {
-      cp_async_wait<1 + PEND>();
+      cp_async_wait<1>();
       __syncwarp();
     } else if (gg == S / 2) {
-      cp_async_wait<PEND>();
+      cp_async_wait<0>();
       __syncwarp();
     }
     const float4* rp = ws.stage + size_t(gg + S * seg) * g.d4;
@@ -801,12 +797,11 @@ struct WarpDist {
       else cpasync_fill_quad<S, false>(g, u_mine, lane, ws);
     }
   }
-  template <int PEND = 0>
   __device__ __forceinline__ float math(const GraphView& g, int lane, WarpSmem& ws) {
     float dot = 0.f;
     if constexpr (uses_tma(NV4))
-      dot = g.d4 == S * C ? cpasync_math<S, C, L2, true, PEND>(g, qv, lane, ws)
-                          : cpasync_math<S, C, L2, false, PEND>(g, qv, lane, ws);
+      dot = g.d4 == S * C ? cpasync_math<S, C, L2, true>(g, qv, lane, ws)
+                          : cpasync_math<S, C, L2, false>(g, qv, lane, ws);
     if constexpr (L2) return dot;
     else return cbase - dot * qinv;
   }
@@ -845,15 +840,10 @@ struct WarpDist {
 // the next vertex explored (2/3 to 4/5 of the iterations in the C2 build), its
 // rows have arrived meanwhile; otherwise the copies are drained and the right
 // rows gathered.  Results never depend on the speculation.
-// DBL (with SPEC; ws.stage2): two stages -- the speculative gather of w goes to the
-// stage the current exploration does not use, issued before the current math, and a
-// miss never waits for a stale speculation before gathering.
-template <class DIST, int TPL, bool COHERENT, bool PREDICT = false, bool SPEC = false,
-          bool DBL = false>
+template <class DIST, int TPL, bool COHERENT, bool PREDICT = false, bool SPEC = false>
 __device__ int warp_search_with(const GraphView& g, DIST& dist, int32_t entry, int l, int e,
                                 WarpSmem& ws, SearchStats& st) {
   static_assert(!(SPEC && PREDICT), "one speculation at a time");
-  static_assert(!DBL || SPEC, "the second stage holds the speculative gather");
   static_assert(!SPEC || TPL == 1, "SPEC gathers one 32-row round");
   const int lane = threadIdx.x & 31;
   uint64_t* sN = ws.sN;
@@ -885,8 +875,6 @@ __device__ int warp_search_with(const GraphView& g, DIST& dist, int32_t entry, i
   int32_t pred_v = -1;      // PREDICT: the vertex predicted after the last lazy check
   int32_t pred_u[TPL];
   int32_t gath_v = -1;      // SPEC: the vertex whose neighbours' rows are in the stage
-  float4* const stage_a = ws.stage;   // DBL: the two stages, and the one holding gath_v's rows
-  float4* spec_st = ws.stage2;
 #if GANNS_PROFILE
   unsigned long long pc[6] = {0, 0, 0, 0, 0, 0};
   unsigned long long p_spec = 0;
@@ -952,31 +940,7 @@ __device__ int warp_search_with(const GraphView& g, DIST& dist, int32_t entry, i
 #pragma unroll
     for (int t = 0; t < TPL; ++t) dist.explore_hint(g, u[t], lane, ws);
     uint64_t key[TPL];
-    if constexpr (SPEC && DBL) {
-      const bool hitg = v == gath_v;
-      float4* const cur = hitg ? spec_st : (spec_st == stage_a ? ws.stage2 : stage_a);
-      float4* const oth = cur == stage_a ? ws.stage2 : stage_a;
-      ws.stage = cur;
-      if (!hitg) dist.fill(g, u[0], lane, ws);
-      float dd;
-      if (w >= 0) {
-        if (!hitg && gath_v >= 0) {   // the stale speculation into oth (older than v's fill) has landed
-          cp_async_wait<2>();
-          __syncwarp();
-        }
-        ws.stage = oth;
-        dist.fill(g, spec_u[0], lane, ws);   // spec_u = w's adjacency row
-        ws.stage = cur;
-        dd = dist.template math<2>(g, lane, ws);
-        gath_v = w;
-        spec_st = oth;
-      } else {
-        dd = dist.template math<0>(g, lane, ws);
-        gath_v = -1;
-      }
-      key[0] = u[0] >= 0 ? mkkey(dd, u[0]) : kKeyInf;
-      st.comps += __popc(__ballot_sync(kFull, u[0] >= 0));
-    } else if constexpr (SPEC) {
+    if constexpr (SPEC) {
 #if GANNS_PROFILE
       // SPEC timers: p_issue = cycles issuing copies (both fills), p_wait = the
       // math incl. its waits, p_rounds = explorations whose rows were gathered ahead
@@ -1195,7 +1159,6 @@ __device__ int warp_search_with(const GraphView& g, DIST& dist, int32_t entry, i
       cp_async_wait<0>();
       __syncwarp();
     }
-  if constexpr (DBL) ws.stage = stage_a;
 #if GANNS_PROFILE
   if (g.prof != nullptr && lane == 0) {
 #pragma unroll
@@ -1219,15 +1182,15 @@ __device__ int warp_search_with(const GraphView& g, DIST& dist, int32_t entry, i
 
 // CPA: the build searches' cp.async gathers (group_distances); SPEC requires it
 template <int NV4, int TPL, bool L2, bool COHERENT, bool PREDICT = false, bool SPEC = false,
-          bool CPA = SPEC, bool DBL = false>
+          bool CPA = SPEC>
 __device__ __forceinline__ int warp_search(const GraphView& g, const float* __restrict__ qrow,
                                            int32_t entry, int l, int e, WarpSmem& ws,
                                            SearchStats& st) {
   static_assert(!SPEC || CPA, "the speculative gather is a cp.async gather");
   WarpDist<NV4, L2, CPA> dist;
   dist.load(g, qrow, threadIdx.x & 31);
-  return warp_search_with<WarpDist<NV4, L2, CPA>, TPL, COHERENT, PREDICT, SPEC, DBL>(
-      g, dist, entry, l, e, ws, st);
+  return warp_search_with<WarpDist<NV4, L2, CPA>, TPL, COHERENT, PREDICT, SPEC>(g, dist, entry, l,
+                                                                               e, ws, st);
 }
 
 // ---------------------------------------------------------------- HNSW
