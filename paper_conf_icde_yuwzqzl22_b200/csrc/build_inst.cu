@@ -296,73 +296,20 @@ phase1_kernel(BuildDev B, int64_t group_size, int64_t g0, int64_t g1,
   if constexpr (GROUP) gdist.post(kCmdExit, lane);
 }
 
-// ------------------------------------------------------------------ K3
-// Phase 2 Step 1 (Alg. 2 lines 10-17; P:285-293) + the counting half of K4, for
-// the vertices [v0, v1) of P_i = [lo, hi).  Fused form (F_ids == nullptr, one GPU):
-// v's row, its E slots and the in-degree counts are written here.  Staged form
-// (multi-GPU build): only the new forward row F (first d_min) is written, to
-// F_ids / F_dists [(v - v0)][d_min]; apply_forward_kernel consumes the F of all of
-// P_i after the exchange.
-// HNSW: the instance that enters through the descent of the upper layers (the
-// plain NSW build's instance carries no descent code)
-template <int NV4, int TPL, bool L2, bool HNSW>
-__global__ void __launch_bounds__(kBuildThreads<NV4>, kBuildMinBlocks<NV4>)
-round_search_kernel(BuildDev B, int64_t lo, int64_t v0, int64_t v1, int32_t* __restrict__ Eu,
-                    float* __restrict__ Ed, int32_t* __restrict__ indeg,
-                    int32_t* __restrict__ touched, int32_t* __restrict__ counters,
-                    int32_t* __restrict__ F_ids, float* __restrict__ F_dists,
-                    const __grid_constant__ CUtensorMap tmap, const UpperLayers U, int layer) {
-  pdl_wait();   // G_0 as the previous round's K5 left it
-  B.g.tmap = &tmap;
-  extern __shared__ __align__(128) uint8_t smem[];
-  // the HNSW instance keeps the one-warp form (its descent is the leader's alone)
-  constexpr bool GROUP = kBuildGroup<NV4> && !HNSW;
-  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int64_t v = v0 + int64_t(blockIdx.x) * kBuildWarps + (kBuildGroup<NV4> ? 0 : w);
-  if (v >= v1) return;
-  if constexpr (kBuildGroup<NV4> && HNSW)
-    if (w != 0) return;
-  WarpSmem ws = carve_build_smem<NV4, TPL>(smem, kBuildGroup<NV4> ? 0 : w, B.l_build, B.g.d4,
-                                           B.wrows_p2);
-  BuildGroupDist<NV4, L2> gdist;
-  if constexpr (GROUP) {
-    gdist.gs = carve_group(smem + build_warp_bytes<NV4, TPL>(B.l_build, B.g.d4, B.wrows_p2));
-    gdist.kc = 0;
-    if (threadIdx.x == 0) mbar_init(ws.mbar, 1);
-    __syncthreads();
-    if (w != 0) {
-      group_helper_loop<(NV4 >= 4 ? NV4 / 4 : 1), L2>(B.g, B.g.X, gdist.gs, ws, w, lane);
-      return;
-    }
-  } else {
-    if (lane == 0) mbar_init(ws.mbar, 1);
-    __syncwarp();
-  }
+// The end of a Phase-2 search of v (Alg. 2 lines 14-17): v.N := first d_min of
+// merge(search result, v.N') (R-C16); fused form: v's row, its E slots and the
+// in-degree counts; staged form: the forward row F only.
+template <int TPL>
+__device__ __forceinline__ void round_finish(const BuildDev& B, int64_t v, int64_t lo, int64_t v0,
+                                             int cnt, const SearchStats& st, WarpSmem& ws, int lane,
+                                             int32_t* __restrict__ Eu, float* __restrict__ Ed,
+                                             int32_t* __restrict__ indeg,
+                                             int32_t* __restrict__ touched,
+                                             int32_t* __restrict__ counters,
+                                             int32_t* __restrict__ F_ids,
+                                             float* __restrict__ F_dists) {
   uint64_t* sN = ws.sN;
   uint64_t* sT = ws.sT;
-  const int d = B.g.d4 * 4;
-  // line 12: v.N := Search(G_0, v, d_min); G_0 = P_0..P_{i-1}, entry = vertex 0;
-  // HNSW (P:371): enter through a greedy descent of the finished upper layers,
-  // kept only if the vertex reached is already in G_0 (R-H2)
-  int32_t entry = 0;
-  if constexpr (HNSW) {
-    if (U.top > layer) {
-      const int32_t c = descend<NV4, TPL, L2, kBuildCpAsync<NV4>>(B.g, U, layer + 1,
-                                                                 B.g.X + size_t(v) * d, ws);
-      entry = c < lo ? c : 0;
-    }
-  }
-  SearchStats st;
-  int cnt;
-  if constexpr (GROUP) {
-    group_new_query(gdist, B.g, B.g.X, v, lane);
-    cnt = warp_search_with<BuildGroupDist<NV4, L2>, TPL, false>(B.g, gdist, entry, B.l_build,
-                                                                B.e_build, ws, st);
-    gdist.post(kCmdExit, lane);
-  } else {
-    cnt = warp_search<NV4, TPL, L2, false, kBuildPredict, kBuildSpec<NV4, TPL>, kBuildCpAsync<NV4>>(
-        B.g, B.g.X + size_t(v) * d, entry, B.l_build, B.e_build, ws, st);
-  }
   add_stats(B.stats, st, lane);
   const int dm = B.d_min;
   const int cs = cnt < dm ? cnt : dm;
@@ -421,6 +368,75 @@ round_search_kernel(BuildDev B, int64_t lo, int64_t v0, int64_t v1, int32_t* __r
       if (atomicAdd(&indeg[u], 1) == 0) touched[atomicAdd(&counters[0], 1)] = u;
     }
   }
+}
+
+// ------------------------------------------------------------------ K3
+// Phase 2 Step 1 (Alg. 2 lines 10-17; P:285-293) + the counting half of K4, for
+// the vertices [v0, v1) of P_i = [lo, hi).  Fused form (F_ids == nullptr, one GPU):
+// v's row, its E slots and the in-degree counts are written here.  Staged form
+// (multi-GPU build): only the new forward row F (first d_min) is written, to
+// F_ids / F_dists [(v - v0)][d_min]; apply_forward_kernel consumes the F of all of
+// P_i after the exchange.
+// HNSW: the instance that enters through the descent of the upper layers (the
+// plain NSW build's instance carries no descent code)
+template <int NV4, int TPL, bool L2, bool HNSW>
+__global__ void __launch_bounds__(kBuildThreads<NV4>, kBuildMinBlocks<NV4>)
+round_search_kernel(BuildDev B, int64_t lo, int64_t v0, int64_t v1, int32_t* __restrict__ Eu,
+                    float* __restrict__ Ed, int32_t* __restrict__ indeg,
+                    int32_t* __restrict__ touched, int32_t* __restrict__ counters,
+                    int32_t* __restrict__ F_ids, float* __restrict__ F_dists,
+                    const __grid_constant__ CUtensorMap tmap, const UpperLayers U, int layer) {
+  pdl_wait();   // G_0 as the previous round's K5 left it
+  B.g.tmap = &tmap;
+  extern __shared__ __align__(128) uint8_t smem[];
+  // the HNSW instance keeps the one-warp form (its descent is the leader's alone)
+  constexpr bool GROUP = kBuildGroup<NV4> && !HNSW;
+  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int64_t v = v0 + int64_t(blockIdx.x) * kBuildWarps + (kBuildGroup<NV4> ? 0 : w);
+  if (v >= v1) return;
+  if constexpr (kBuildGroup<NV4> && HNSW)
+    if (w != 0) return;
+  WarpSmem ws = carve_build_smem<NV4, TPL>(smem, kBuildGroup<NV4> ? 0 : w, B.l_build, B.g.d4,
+                                           B.wrows_p2);
+  BuildGroupDist<NV4, L2> gdist;
+  if constexpr (GROUP) {
+    gdist.gs = carve_group(smem + build_warp_bytes<NV4, TPL>(B.l_build, B.g.d4, B.wrows_p2));
+    gdist.kc = 0;
+    if (threadIdx.x == 0) mbar_init(ws.mbar, 1);
+    __syncthreads();
+    if (w != 0) {
+      group_helper_loop<(NV4 >= 4 ? NV4 / 4 : 1), L2>(B.g, B.g.X, gdist.gs, ws, w, lane);
+      return;
+    }
+  } else {
+    if (lane == 0) mbar_init(ws.mbar, 1);
+    __syncwarp();
+  }
+  const int d = B.g.d4 * 4;
+  // line 12: v.N := Search(G_0, v, d_min); G_0 = P_0..P_{i-1}, entry = vertex 0;
+  // HNSW (P:371): enter through a greedy descent of the finished upper layers,
+  // kept only if the vertex reached is already in G_0 (R-H2)
+  int32_t entry = 0;
+  if constexpr (HNSW) {
+    if (U.top > layer) {
+      const int32_t c = descend<NV4, TPL, L2, kBuildCpAsync<NV4>>(B.g, U, layer + 1,
+                                                                 B.g.X + size_t(v) * d, ws);
+      entry = c < lo ? c : 0;
+    }
+  }
+  SearchStats st;
+  int cnt;
+  if constexpr (GROUP) {
+    group_new_query(gdist, B.g, B.g.X, v, lane);
+    cnt = warp_search_with<BuildGroupDist<NV4, L2>, TPL, false>(B.g, gdist, entry, B.l_build,
+                                                                B.e_build, ws, st);
+    gdist.post(kCmdExit, lane);
+  } else {
+    cnt = warp_search<NV4, TPL, L2, false, kBuildPredict, kBuildSpec<NV4, TPL>, kBuildCpAsync<NV4>>(
+        B.g, B.g.X + size_t(v) * d, entry, B.l_build, B.e_build, ws, st);
+  }
+  round_finish<TPL>(B, v, lo, v0, cnt, st, ws, lane, Eu, Ed, indeg, touched, counters, F_ids,
+                    F_dists);
 }
 
 // Staged form, after the exchange: the F of every v in P_i = [lo, hi) becomes v's

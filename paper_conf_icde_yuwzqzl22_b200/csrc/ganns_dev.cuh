@@ -797,6 +797,11 @@ struct WarpDist {
       else cpasync_fill_quad<S, false>(g, u_mine, lane, ws);
     }
   }
+  // a fill whose rows are not needed (a missed speculation) completes
+  __device__ __forceinline__ void drain(WarpSmem&) {
+    cp_async_wait<0>();
+    __syncwarp();
+  }
   __device__ __forceinline__ float math(const GraphView& g, int lane, WarpSmem& ws) {
     float dot = 0.f;
     if constexpr (uses_tma(NV4))
@@ -948,10 +953,7 @@ __device__ int warp_search_with(const GraphView& g, DIST& dist, int32_t entry, i
       ws.p_rounds += v == gath_v ? 1 : 0;
 #endif
       if (v != gath_v) {   // not gathered ahead: drain the speculative copies, gather
-        if (gath_v >= 0) {
-          cp_async_wait<0>();
-          __syncwarp();
-        }
+        if (gath_v >= 0) dist.drain(ws);
         dist.fill(g, u[0], lane, ws);
       }
 #if GANNS_PROFILE
@@ -1155,10 +1157,7 @@ __device__ int warp_search_with(const GraphView& g, DIST& dist, int32_t entry, i
     GANNS_PROF_MARK(kProfMerge);
   }
   if constexpr (SPEC)
-    if (gath_v >= 0) {   // the last speculation's copies land before the stage is reused
-      cp_async_wait<0>();
-      __syncwarp();
-    }
+    if (gath_v >= 0) dist.drain(ws);   // the last speculation's copies land before the stage is reused
 #if GANNS_PROFILE
   if (g.prof != nullptr && lane == 0) {
 #pragma unroll
