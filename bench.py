@@ -464,6 +464,8 @@ def roofline(alg_bytes, launch_s, dram, launches, peak, peak_kind, kernel, durat
     else:
         r.update(achieved=round(alg, 1), frac=round(alg / peak, 4), traffic=None,
                  achieved_kind=f"algorithmic (DRAM counters unavailable: {dram['error']})")
+    # also against the B200 HBM3e specification (~8 TB/s)
+    r["frac_of_spec_8TBps"] = round(r["achieved"] / 8000.0, 4)
     return r
 
 
