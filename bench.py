@@ -213,7 +213,7 @@ class BenchIndex:
         if self.hnsw:
             levels = syn.hnsw_levels(Xd.shape[0], cfg.degree // 2, 1)
             self.idx = g.build_hnsw(Xd, levels, metric=cfg.metric, degree=cfg.degree,
-                                    l_build=l_build)
+                                    l_build=l_build, l_local=min(l_local, l_build))
             self.graph = self.idx.base
             self.build_stats = self.idx.build_stats
         else:
@@ -714,8 +714,7 @@ def run_ours(args):
         "build_seconds": round(build_s, 4),
         "build_seconds_all": [round(x, 4) for x in build_all],
         "build_params": {"degree": cfg.degree, "d_min": cfg.degree // 2, "l_build": args.l_build,
-                         "l_local": (None if index.hnsw else min(args.l_local, args.l_build) or
-                                     args.l_build),
+                         "l_local": min(args.l_local, args.l_build) or args.l_build,
                          "group_size": "auto"},
         "build": {"iterations": b_iters, "distance_computations": b_comps,
                   "searches": b_searches, "rounds": b_rounds,

@@ -259,7 +259,8 @@ GANNS_API void ganns_graph_free(ganns_graph *g);
  * from the vertex reached. */
 typedef struct ganns_hnsw ganns_hnsw;
 
-/* ganns_build_hnsw -- as ganns_build, plus
+/* ganns_build_hnsw -- as ganns_build (p->max_rounds and p->stop_after_phase1 are
+ * ignored; p->l_local applies to every layer's Phase 1, R-C13), plus
  *   levels_host  host int8 [n], level of every point, 0 <= level < 16.
  * Syncs.  The index keeps a device copy of the rows of the upper-layer points. */
 GANNS_API int ganns_build_hnsw(const float *points, int64_t n, int d, int metric, int degree,

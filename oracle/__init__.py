@@ -59,8 +59,8 @@ def lib():
         _lib.ora_merge_topk.argtypes = [P, P, i32, i64, i32, P, P]
         _lib.ora_knn_descent.argtypes = [P, i64, i32, i32, i32, P, i32, P, P, P]
         _lib.ora_knn_descent.restype = ct.c_int
-        _lib.ora_hnsw_build.argtypes = [P, i64, i32, i32, P, i32, i32, i32, i32, i64, P, P, P,
-                                        P, P]
+        _lib.ora_hnsw_build.argtypes = [P, i64, i32, i32, P, i32, i32, i32, i32, i32, i64, P, P,
+                                        P, P, P]
         _lib.ora_hnsw_search.argtypes = [P, P, i32, P, P, i64, i32, P, i32, i32, P, i64, i32,
                                          i32, i32, P, P, P, P, P]
         for f in ("ora_hnsw_build", "ora_hnsw_search", "ora_merge_topk", "ora_search_one", "ora_search_batch", "ora_alg1", "ora_bruteforce",
@@ -218,10 +218,12 @@ def merge_topk(ids, dists):
     return oi, od
 
 
-def hnsw_build(X, levels, d_min, d_max, group_size, l_build=64, e_build=0, metric="l2"):
+def hnsw_build(X, levels, d_min, d_max, group_size, l_build=64, e_build=0, metric="l2",
+               l_local=0):
     """HNSW (Section IV-D).  Returns dict(perm, layer_n, upper, layer0):
     perm[new] = old; layer_n[j] = |layer j|; upper[j] (j >= 1) = [n_j, d_max] adjacency
-    in shuffled ids; layer0 = [n, d_max] adjacency in original ids."""
+    in shuffled ids; layer0 = [n, d_max] adjacency in original ids.  l_local (0 =
+    l_build): list length of every layer's Phase-1 searches (R-C13)."""
     X = _f32(X)
     levels = np.ascontiguousarray(levels, dtype=np.int8)
     n = X.shape[0]
@@ -233,7 +235,7 @@ def hnsw_build(X, levels, d_min, d_max, group_size, l_build=64, e_build=0, metri
     upper = np.empty(max(1, sum(cnt[1:]) * d_max), np.int32)
     layer0 = np.empty((n, d_max), np.int32)
     _check(lib().ora_hnsw_build(_p(X), n, X.shape[1], METRICS[metric], _p(levels), d_min, d_max,
-                                l_build, e_build, group_size, _p(perm), _p(layer_n),
+                                l_build, e_build, l_local, group_size, _p(perm), _p(layer_n),
                                 ct.byref(nl), _p(upper), _p(layer0)))
     ups, off = {}, 0
     for j in range(1, nl.value):

@@ -509,13 +509,15 @@ class Hnsw:
 
 def build_hnsw(points: torch.Tensor, levels: np.ndarray, metric: str = "l2", degree: int = 32,
                d_min: int = 0, l_build: int = 0, e_build: int = 0, group_size: int = 0,
-               stream=None) -> Hnsw:
+               stream=None, l_local: int = 0) -> Hnsw:
     """HNSW construction: Algorithm 2 per layer, top-down.  `levels`
-    int8 [n] (e.g. ganns_synth.hnsw_levels)."""
+    int8 [n] (e.g. ganns_synth.hnsw_levels).  l_local (0 = l_build): list length of
+    every layer's Phase-1 searches (R-C13)."""
     points = _dev_f32(points, "points")
     levels = np.ascontiguousarray(levels, dtype=np.int8)
     st = (ct.c_uint64 * 4)()
-    p = _BuildParams(d_min, l_build, e_build, group_size, 0, 0, ct.cast(st, ct.POINTER(ct.c_uint64)))
+    p = _BuildParams(d_min, l_build, e_build, group_size, 0, 0, ct.cast(st, ct.POINTER(ct.c_uint64)),
+                     l_local)
     h = ct.c_void_p()
     with torch.cuda.device(points.device):
         _check(_lib.ganns_build_hnsw(ct.c_void_p(points.data_ptr()), points.shape[0],

@@ -765,6 +765,8 @@ int ganns_build_hnsw(const float* points, int64_t n, int d, int metric, int degr
   if (d_min > degree || d_min >= n) return fail(GANNS_EINVAL, "bad d_min");
   if (l_build < d_min || l_build > 1024) return fail(GANNS_EINVAL, "l_build must be in [d_min, 1024]");
   if (e_build < 1 || e_build > l_build) return fail(GANNS_EINVAL, "e_build must be in [1, l_build]");
+  const int l_local = p && p->l_local > 0 ? p->l_local : l_build;
+  if (l_local < d_min || l_local > l_build) return fail(GANNS_EINVAL, "l_local must be in [d_min, l_build]");
   // (1) shuffled ids: points by level descending, ties by id (stable counting sort)
   int top = 0;
   for (int64_t v = 0; v < n; ++v) {
@@ -828,8 +830,8 @@ int ganns_build_hnsw(const float* points, int64_t n, int d, int metric, int degr
     a.d_min = d_min;
     a.l_build = l_build;
     a.e_build = e_build;
-    a.l_local = l_build;   // HNSW layers: Phase 1 at l_build (the oracle's HNSW has no l_local)
-    a.e_local = e_build;
+    a.l_local = l_local;   // every layer's Phase-1 searches (R-C13)
+    a.e_local = std::min(e_build, l_local);
     int64_t S = p && p->group_size > 0 ? p->group_size : 0;
     if (S == 0) S = auto_group_size(layer_n[j]);
     a.group_size = std::max<int64_t>(1, std::min<int64_t>(S, layer_n[j]));

@@ -20,19 +20,23 @@ def cu(a):
     return torch.from_numpy(np.ascontiguousarray(a)).to(DEV)
 
 
-@pytest.mark.parametrize("n,degree,l_build,s,metric,seed", [
-    (3000, 16, 32, 128, "l2", 1),
-    (2500, 32, 64, 256, "l2", 2),
-    (2000, 16, 32, 100, "ip", 3),
+@pytest.mark.parametrize("n,degree,l_build,s,metric,seed,l_local", [
+    (3000, 16, 32, 128, "l2", 1, 0),
+    (2500, 32, 64, 256, "l2", 2, 0),
+    (2000, 16, 32, 100, "ip", 3, 0),
+    (2500, 32, 64, 256, "l2", 4, 24),    # every layer's Phase 1 at l_local (R-C13)
+    (2000, 16, 48, 100, "ip", 5, 16),
 ])
-def test_hnsw_build_and_search_parity(n, degree, l_build, s, metric, seed):
+def test_hnsw_build_and_search_parity(n, degree, l_build, s, metric, seed, l_local):
     cfg = syn.with_size(syn.CONFIGS["C1"], n=n, nq=100)
     X, Q = syn.points(cfg), syn.queries(cfg)
     if metric == "ip":
         X, Q = X - 128.0, Q - 128.0
     levels = syn.hnsw_levels(n, degree // 2, seed)
-    ref = oracle.hnsw_build(X, levels, degree // 2, degree, s, l_build=l_build, metric=metric)
-    idx = g.build_hnsw(cu(X), levels, metric=metric, degree=degree, l_build=l_build, group_size=s)
+    ref = oracle.hnsw_build(X, levels, degree // 2, degree, s, l_build=l_build, metric=metric,
+                            l_local=l_local)
+    idx = g.build_hnsw(cu(X), levels, metric=metric, degree=degree, l_build=l_build, group_size=s,
+                       l_local=l_local)
     torch.cuda.synchronize()
     assert idx.nlayers == len(ref["layer_n"]) and idx.layer_n == ref["layer_n"].tolist()
     assert (idx.perm() == ref["perm"]).all()

@@ -62,7 +62,7 @@ def test_c4_instance_hnsw_fused_l288_integer_ip_bitexact():
     cfg, X, Q = _c4_like(100_000, "ip")
     Xd = cu(X)
     levels = syn.hnsw_levels(len(X), cfg.degree // 2, 1)
-    idx = g.build_hnsw(Xd, levels, metric="ip", degree=cfg.degree, l_build=128)
+    idx = g.build_hnsw(Xd, levels, metric="ip", degree=cfg.degree, l_build=128, l_local=32)
     assert idx.nlayers >= 3
     ids, dists, st, ds = g.hnsw_search(idx, Xd, cu(Q), cfg.k, 288, stats=True,
                                        descent_stats=True)   # one launch
@@ -85,7 +85,7 @@ def test_c4_instance_hnsw_fused_l288_cosine():
     cfg, X, Q = _c4_like(100_000, "cosine")
     Xd = cu(X)
     levels = syn.hnsw_levels(len(X), cfg.degree // 2, 1)
-    idx = g.build_hnsw(Xd, levels, metric="cosine", degree=cfg.degree, l_build=128)
+    idx = g.build_hnsw(Xd, levels, metric="cosine", degree=cfg.degree, l_build=128, l_local=32)
     ids, dists = g.hnsw_search(idx, Xd, cu(Q), cfg.k, 288)
     ids, dists = ids.cpu().numpy(), dists.cpu().numpy()
     h = oracle_index(idx)

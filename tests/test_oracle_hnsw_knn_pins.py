@@ -11,6 +11,7 @@
   sets and lexsort.
 """
 import numpy as np
+import pytest
 
 import oracle
 import ganns_synth as syn
@@ -105,11 +106,13 @@ def _search1(nbr, Y, q, k, l, e, entry):
     return [(float(dd), int(i)) for dd, i in zip(dists[0], ids[0]) if i >= 0]
 
 
-def _alg2_restated(Y, d_min, d_max, S, l_b, entry_of):
+def _alg2_restated(Y, d_min, d_max, S, l_b, entry_of, l_loc=0):
     """Algorithm 2 in plain Python lists: Phase 1 local graphs with
-    sorted truncated back-insertion; Phase 2 rounds: search G_0 from
-    entry_of(v, lo), first d_min of (S u N'(v)) (R-C16), v's row replaced
-    (R-C15), E sorted by (u, dist, v) (R-C17) merged into u's row keeping d_max."""
+    sorted truncated back-insertion, searched at list length l_loc (0 = l_b,
+    R-C13); Phase 2 rounds: search G_0 from entry_of(v, lo), first d_min of
+    (S u N'(v)) (R-C16), v's row replaced (R-C15), E sorted by (u, dist, v) (R-C17)
+    merged into u's row keeping d_max."""
+    l_p1 = l_loc or l_b
     n = len(Y)
     rows = [[] for _ in range(n)]                 # sorted (dist, id) lists
 
@@ -124,7 +127,7 @@ def _alg2_restated(Y, d_min, d_max, S, l_b, entry_of):
     for g in range(ng):
         lo, hi = g * S, min(n, (g + 1) * S)
         for v in range(lo, hi):
-            F = [] if v == lo else _search1(adj(), Y, Y[v], d_min, l_b, 0, lo)[:d_min]
+            F = [] if v == lo else _search1(adj(), Y, Y[v], d_min, l_p1, 0, lo)[:d_min]
             rows[v] = list(F)
             gp[v] = list(F)
             for dist, u in F:
@@ -149,15 +152,20 @@ def _alg2_restated(Y, d_min, d_max, S, l_b, entry_of):
     return adj()
 
 
-def test_hnsw_build_matches_restated_algorithm2_with_descent_entries():
+@pytest.mark.parametrize("l_loc", [0, 3])
+def test_hnsw_build_matches_restated_algorithm2_with_descent_entries(l_loc):
     """Non-exact regime (l_build = 6 << n).  Layers are built top-down; a Phase-2
     search of layer j enters at the greedy descent of the finished layers above
     (l = e = 1 from shuffled id 0), or at vertex 0 when that vertex is not yet in
-    G_0 (R-H2).  Both branches occur in this instance."""
+    G_0 (R-H2).  Both branches occur in this instance.  l_loc: every layer's Phase 1
+    at list length 3 (R-C13), which changes the index."""
     n, d_min, d_max, S, l_b = 420, 3, 6, 40, 6
     X = syn.random_int_points(n, 8, 0, 15, 77)
     levels = syn.hnsw_levels(n, d_min, 5)
-    h = oracle.hnsw_build(X, levels, d_min, d_max, group_size=S, l_build=l_b)
+    h = oracle.hnsw_build(X, levels, d_min, d_max, group_size=S, l_build=l_b, l_local=l_loc)
+    if l_loc:
+        h0 = oracle.hnsw_build(X, levels, d_min, d_max, group_size=S, l_build=l_b)
+        assert (h["layer0"] != h0["layer0"]).any()
     perm = h["perm"]
     assert perm.tolist() == sorted(range(n), key=lambda v: (-levels[v], v))
     L = int(levels.max()) + 1
@@ -178,7 +186,7 @@ def test_hnsw_build_matches_restated_algorithm2_with_descent_entries():
                 return 0
             used["descent"] += cur != 0
             return cur
-        built[j] = _alg2_restated(Xp[:sizes[j]], d_min, d_max, S, l_b, entry_of)
+        built[j] = _alg2_restated(Xp[:sizes[j]], d_min, d_max, S, l_b, entry_of, l_loc)
         if j >= 1:
             assert (h["upper"][j] == built[j]).all(), f"layer {j}"
     assert used["fallback"] > 0 and used["descent"] > 0, used
