@@ -469,6 +469,31 @@ def roofline(alg_bytes, launch_s, dram, launches, peak, peak_kind, kernel, durat
     return r
 
 
+def build_phase_split(torch, g, cfg, Xd, l_build, l_local):
+    """Phase 1 and the serial Phase-2 rounds of Algorithm 2 timed apart on
+    the GPU clock -- one extra build through the staged ABI (ganns_build_begin ...,
+    the same kernels; a round's searches then write F and an apply kernel writes the
+    rows), CUDA events around Phase 1 and around all rounds."""
+    b = g.StagedBuild(Xd, metric=cfg.metric, degree=cfg.degree, l_build=l_build,
+                      l_local=min(l_local, l_build))
+    _, G, _, _ = b.info()
+    ev = [torch.cuda.Event(enable_timing=True) for _ in range(3)]
+    ev[0].record()
+    b.phase1(0, G)
+    ev[1].record()
+    for i in range(1, G):
+        v0, v1 = b.group_rows(i, i + 1)
+        b.round_apply(i, *b.round_search(i, v0, v1))
+    ev[2].record()
+    ev[2].synchronize()
+    gr = b.finish()
+    del gr
+    p1, p2 = ev[0].elapsed_time(ev[1]) / 1e3, ev[1].elapsed_time(ev[2]) / 1e3
+    return {"phase1_s": round(p1, 4), "phase2_s": round(p2, 4), "rounds": G - 1,
+            "round_ms_mean": round(p2 / max(1, G - 1) * 1e3, 4),
+            "method": "staged ABI, CUDA events on the build's stream (GPU clock)"}
+
+
 def cpu_model():
     try:
         with open("/proc/cpuinfo") as f:
@@ -592,6 +617,8 @@ def run_ours(args):
         build_all.append(time.perf_counter() - t0)
     build_s = statistics.median(build_all)
     b_iters, b_comps, b_searches, b_rounds = index.build_stats
+    phase_split = None if index.hnsw else build_phase_split(torch, g, cfg, Xd, args.l_build,
+                                                            args.l_local)
 
     # ---- (l, e) operating point over every query the timed steps search (see
     # select_operating_point); candidates timed as the steps are (pipelined)
@@ -718,7 +745,8 @@ def run_ours(args):
                          "group_size": "auto"},
         "build": {"iterations": b_iters, "distance_computations": b_comps,
                   "searches": b_searches, "rounds": b_rounds,
-                  "alg_GBps": round((4 * d * b_comps + 4 * cfg.degree * b_iters) / build_s / 1e9, 1)},
+                  "alg_GBps": round((4 * d * b_comps + 4 * cfg.degree * b_iters) / build_s / 1e9, 1),
+                  "phase_split": phase_split},
         "e2e": {"value": round(e2e_qps, 1), "unit": "queries/s",
                 "h2d_bytes_per_step": int(Qhs[0].numel() * 4),
                 "d2h_bytes_per_step": int((hi - lo) * k * 8),
