@@ -223,6 +223,138 @@ knn_propose_kernel(const float* __restrict__ X, int64_t n, int d4, int K,
   }
 }
 
+// Register-tiled form of knn_propose_kernel (same proposals, same arithmetic per
+// pair): the rows of S(v) are staged by cp.async (all in flight at once), then the
+// m x m pair distances are computed in 4 passes of 4 x 8 tiles per lane -- lane
+// (ga = lane % 4, gb = lane / 4) owns a-rows ga + 4 i + 16 p and b-rows gb + 8 j --
+// so each staged float4 is loaded once per tile instead of once per pair (the
+// one-pair-per-lane form was bound by shared-memory bandwidth: ~4 MB of LDS per v
+// at m = 64, d = 128).  Loads are conflict-free with the padded row pitch.
+#ifndef GANNS_KNN_TILED
+#define GANNS_KNN_TILED 1
+#endif
+__host__ __device__ constexpr size_t knn_tiled_warp_smem(int d4) {
+  return size_t(64) * (d4 + 1) * 16 + 64 * 4 + 64 * 8;
+}
+template <bool L2>
+__global__ void __launch_bounds__(kKnnWarps * 32)
+knn_propose_tiled_kernel(const float* __restrict__ X, int64_t n, int d4, int K,
+                         const int32_t* __restrict__ ids, const float* __restrict__ dists,
+                         const int32_t* __restrict__ rev, int32_t* __restrict__ Pa,
+                         float* __restrict__ Pd, int32_t* __restrict__ Pb,
+                         unsigned long long* __restrict__ pcount, unsigned long long cap,
+                         int* __restrict__ overflow) {
+  extern __shared__ __align__(16) uint8_t smem[];
+  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int pitch4 = d4 + 1;
+  uint8_t* base = smem + size_t(w) * knn_tiled_warp_smem(d4);
+  float4* stage = reinterpret_cast<float4*>(base);
+  int32_t* sS = reinterpret_cast<int32_t*>(base + size_t(64) * pitch4 * 16);
+  uint64_t* sW = reinterpret_cast<uint64_t*>(sS + 64);
+  const float4* X4 = reinterpret_cast<const float4*>(X);
+  const int ga = lane & 3, gb = lane >> 2;
+  const int64_t nwarps = int64_t(gridDim.x) * kKnnWarps;
+  for (int64_t v = int64_t(blockIdx.x) * kKnnWarps + w; v < n; v += nwarps) {
+    // S(v): forward ids, then the reverse ids not already present (R-K2)
+    const int32_t f = lane < K ? ids[size_t(v) * K + lane] : -1;
+    int32_t r = lane < K ? rev[size_t(v) * K + lane] : -1;
+    for (int j = 0; j < K; ++j)
+      if (__shfl_sync(kFull, f, j) == r) r = -1;
+    const unsigned fm = __ballot_sync(kFull, f >= 0), rm = __ballot_sync(kFull, r >= 0);
+    const int nf = __popc(fm), m = nf + __popc(rm);
+    if (f >= 0) sS[__popc(fm & lanemask_lt())] = f;
+    if (r >= 0) sS[nf + __popc(rm & lanemask_lt())] = r;
+    __syncwarp();
+    // stage the m rows: every copy in flight at once
+    for (int t = 0; t < m; ++t) {
+      const float4* src = X4 + size_t(sS[t]) * d4;
+      float4* dst = stage + size_t(t) * pitch4;
+      for (int c = lane; c < d4; c += 32)
+        asm volatile("cp.async.ca.shared.global [%0], [%1], 16;" ::"r"(smem_u32(dst + c)), "l"(src + c)
+                     : "memory");
+    }
+    asm volatile("cp.async.commit_group;" ::: "memory");
+    // the K-th key of every a (what a proposal must beat)
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {
+      const int t = lane + 32 * h;
+      uint64_t wk = kKeyInf;
+      if (t < m) {
+        const int32_t a = sS[t];
+        const int32_t wid = ids[size_t(a) * K + K - 1];
+        wk = wid >= 0 ? mkkey(dists[size_t(a) * K + K - 1], wid) : kKeyInf;
+      }
+      sW[t] = wk;
+    }
+    asm volatile("cp.async.wait_all;" ::: "memory");
+    __syncwarp();
+    for (int p = 0; p * 16 < m; ++p) {
+      uint64_t acc[4][8];
+#pragma unroll
+      for (int i = 0; i < 4; ++i)
+#pragma unroll
+        for (int j = 0; j < 8; ++j) acc[i][j] = 0;
+      int ta[4], tb[8];
+#pragma unroll
+      for (int i = 0; i < 4; ++i) ta[i] = min(ga + 4 * i + 16 * p, 63);
+#pragma unroll
+      for (int j = 0; j < 8; ++j) tb[j] = gb + 8 * j;
+      for (int c = 0; c < d4; ++c) {
+        float4 ra[4], rb[8];
+#pragma unroll
+        for (int i = 0; i < 4; ++i) ra[i] = stage[size_t(ta[i]) * pitch4 + c];
+#pragma unroll
+        for (int j = 0; j < 8; ++j) rb[j] = stage[size_t(tb[j]) * pitch4 + c];
+#pragma unroll
+        for (int i = 0; i < 4; ++i)
+#pragma unroll
+          for (int j = 0; j < 8; ++j) acc[i][j] = accum4<L2>(acc[i][j], ra[i], rb[j]);
+      }
+      // proposals of this pass: a = S[t] -> b = S[u] where the key beats a's K-th
+      unsigned pm = 0;
+      float dd[4][8];
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        const int t = ga + 4 * i + 16 * p;
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+          const int u = tb[j];
+          dd[i][j] = L2 ? hsum2(acc[i][j]) : 0.f - hsum2(acc[i][j]);
+          const bool ok = t < m && u < m && t != u && mkkey(dd[i][j], sS[u]) < sW[t];
+          pm |= ok ? 1u << (i * 8 + j) : 0u;
+        }
+      }
+      const int mine = __popc(pm);
+      int incl = mine;
+#pragma unroll
+      for (int off = 1; off < 32; off <<= 1) {
+        const int y = __shfl_up_sync(kFull, incl, off);
+        if (lane >= off) incl += y;
+      }
+      const int total = __shfl_sync(kFull, incl, 31);
+      if (total == 0) continue;
+      unsigned long long at0 = 0;
+      if (lane == 0) at0 = atomicAdd(pcount, (unsigned long long)total);
+      unsigned long long at = __shfl_sync(kFull, at0, 0) + (incl - mine);
+#pragma unroll
+      for (int i = 0; i < 4; ++i)
+#pragma unroll
+        for (int j = 0; j < 8; ++j)
+          if (pm & (1u << (i * 8 + j))) {
+            if (at < cap) {
+              Pa[at] = sS[ga + 4 * i + 16 * p];
+              Pd[at] = dd[i][j];
+              Pb[at] = sS[tb[j]];
+            } else {
+              *overflow = 1;
+            }
+            ++at;
+          }
+    }
+    __syncwarp();
+  }
+}
+
 __global__ void prop_scatter_kernel(const int32_t* __restrict__ Pa, const float* __restrict__ Pd,
                                     const int32_t* __restrict__ Pb, const unsigned long long* pcount,
                                     const int64_t* __restrict__ off, int32_t* __restrict__ fill,
@@ -327,10 +459,13 @@ static int knn_t(const float* X, int64_t n, int d, int K, const int32_t* init_de
   knn_init_kernel<L2><<<grid, 128, 0, s>>>(X, n, d4, K, init_dev, out_ids, dists.p);
   count_launch();
   KNN_TRY(cudaGetLastError());
-  const size_t smem = size_t(kKnnWarps) * knn_warp_smem(d4);
+  const bool tiled = GANNS_KNN_TILED != 0;
+  const size_t smem = size_t(kKnnWarps) * (tiled ? knn_tiled_warp_smem(d4) : knn_warp_smem(d4));
   if (smem > 227 * 1024) return fail(GANNS_ENOTSUP, "knn: staged rows exceed shared memory");
   KNN_TRY(cudaFuncSetAttribute(knn_propose_kernel<L2>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                int(smem)));
+  KNN_TRY(cudaFuncSetAttribute(knn_propose_tiled_kernel<L2>,
+                               cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem)));
   int it = 0;
   unsigned long long h[3] = {0, 0, 0};
   for (; it < max_iters;) {
@@ -341,9 +476,13 @@ static int knn_t(const float* X, int64_t n, int d, int K, const int32_t* init_de
     rev_scatter_kernel<<<grid, 256, 0, s>>>(out_ids, dists.p, n, K, off.p, fill.p, seg.p);
     rev_select_kernel<<<grid, 128, 0, s>>>(n, K, cnt.p, fill.p, off.p, seg.p, rev.p);
     // proposals
-    knn_propose_kernel<L2><<<grid, kKnnWarps * 32, smem, s>>>(X, n, d4, K, out_ids, dists.p, rev.p,
-                                                           Pa.p, Pd.p, Pb.p, counters.p + 1, cap,
-                                                           overflow.p);
+    if (tiled)
+      knn_propose_tiled_kernel<L2><<<grid, kKnnWarps * 32, smem, s>>>(
+          X, n, d4, K, out_ids, dists.p, rev.p, Pa.p, Pd.p, Pb.p, counters.p + 1, cap, overflow.p);
+    else
+      knn_propose_kernel<L2><<<grid, kKnnWarps * 32, smem, s>>>(X, n, d4, K, out_ids, dists.p,
+                                                             rev.p, Pa.p, Pd.p, Pb.p,
+                                                             counters.p + 1, cap, overflow.p);
     // bucket by a, merge
     KNN_TRY(cudaMemsetAsync(counters.p, 0, sizeof(unsigned long long), s));
     prop_count_kernel<<<grid, 256, 0, s>>>(Pa.p, counters.p + 1, cnt.p);
