@@ -838,7 +838,7 @@ struct WarpDist {
 // predicted -- the smallest surviving neighbour always enters N, so it is next
 // whenever it precedes the second unexplored entry w -- and its adjacency row is
 // loaded while the sort and merge run.  Results never depend on the prediction.
-// SPEC (build searches with ws.cpasync, d_max <= 32): right after an exploration's
+// SPEC (build searches with the cp.async gather, CPA; d_max <= 32): right after an exploration's
 // distance math, the rows of w (the second unexplored entry, whose adjacency row
 // the speculation loads with v's) are gathered into the stage -- the stage is
 // idle during the lazy check, sort and merge (T lives outside it).  When w is
