@@ -70,7 +70,7 @@ static cudaError_t launch_pdl(void (*k)(KArgs...), unsigned grid, unsigned block
   return cudaLaunchKernelEx(&cfg, k, static_cast<KArgs>(args)...);
 }
 
-constexpr int kBuildWarps = 1;
+constexpr int kBuildWarps = 1;   // one warp per CTA spreads the latency-bound build searches over all SMs
 // d > 256 (GANNS_BUILD_GROUP): a build search is run by a warp group, as the wide
 // batched search (search_group.cuh): warp 0 runs the loop, all kGroupWarps warps
 // reduce their column slices of each staged row -- one CTA of kGroupWarps warps
@@ -88,7 +88,7 @@ constexpr int kBuildThreads = kBuildGroup<NV4> ? kGroupWarps * 32 : kBuildWarps 
 template <int NV4>
 constexpr int kBuildMinBlocks = kBuildGroup<NV4> ? kGroupMinBlocks : 12;
 template <int NV4, bool L2>
-using BuildGroupDist = GroupDist<(NV4 >= 4 ? NV4 / 4 : 1), L2>;   // one warp per CTA spreads the latency-bound build searches over all SMs
+using BuildGroupDist = GroupDist<(NV4 >= 4 ? NV4 / 4 : 1), L2>;
 #ifndef GANNS_BUILD_PREDICT
 #define GANNS_BUILD_PREDICT 0
 #endif
@@ -99,7 +99,7 @@ using BuildGroupDist = GroupDist<(NV4 >= 4 ? NV4 / 4 : 1), L2>;   // one warp pe
 // warp-min and load sit on the chain and the hidden adjacency latency is small (the
 // adjacency rows mostly hit L2)
 constexpr bool kBuildPredict = GANNS_BUILD_PREDICT != 0;
-// The build searches' stage is filled by cp.async (ganns_dev.cuh: cpasync_fill) for
+// The build searches' stage is filled by cp.async (ganns_dev.cuh: cpasync_fill_quad) for
 // d <= 256, and (d_max <= 32) the next exploration's rows are gathered
 // speculatively while the lazy check, sort and merge run (warp_search_with, SPEC).
 // A build search is a latency chain: a Phase-2 round lasts as long as its slowest
