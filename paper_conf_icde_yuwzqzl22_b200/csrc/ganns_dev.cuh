@@ -596,7 +596,7 @@ __device__ __forceinline__ void cpasync_fill_quad(const GraphView& g, int32_t u_
   }
 }
 
-// the math over a stage filled by cpasync_fill (its two groups must be this
+// the math over a stage filled by cpasync_fill_quad (its two groups must be this
 // thread's last two commits; any older group is waited for as well).  The stage
 // loads are plain (not lds128_ordered): ptxas may hoist a half's 4 x C loads ahead
 // of its math -- the build searches are latency-bound and have registers to spare
@@ -709,7 +709,7 @@ __device__ __forceinline__ float wide_dot(const GraphView& g, const float4 (&qv)
   return dres;
 }
 
-// CPA (build searches, d <= 256): the stage is filled by cp.async (cpasync_fill),
+// CPA (build searches, d <= 256): the stage is filled by cp.async (cpasync_fill_quad),
 // one round of <= 32 rows
 template <int NV4, bool L2, bool CPA = false>
 __device__ __forceinline__ float group_distances(const GraphView& g,
