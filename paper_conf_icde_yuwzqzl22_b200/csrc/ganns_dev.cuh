@@ -189,6 +189,11 @@ constexpr int kWideStageRows = 8;   // d > 256: rows per TMA round (4 rounds per
 #ifndef GANNS_SKIP_LB
 #define GANNS_SKIP_LB 1
 #endif
+// GANNS_LB_PRELOAD: load N's l-th key and the lazy check's first probes before the
+// bulk-distance gather (their latency hides under it)
+#ifndef GANNS_LB_PRELOAD
+#define GANNS_LB_PRELOAD 1
+#endif
 #ifndef GANNS_PREFETCH_R2
 #define GANNS_PREFETCH_R2 0
 #endif
@@ -941,6 +946,23 @@ __device__ int warp_search_with(const GraphView& g, DIST& dist, int32_t entry, i
     if (__ballot_sync(kFull, u[0] >= 0) == 0xdeadbeefu) st.merged += 0;   // waits for the row
     GANNS_PROF_MARK(kProfExplore);
 #endif
+    // the lazy check's key-independent loads, issued before the gather so their
+    // latency hides under it (the latency-bound build searches, SPEC; the batched
+    // search measured 1.5-2.5 % slower with it): N's l-th key and the first 4-ary
+    // step's three probes (N's distances do not change until the merge; the
+    // explored flag set by the locate step is masked off)
+    constexpr bool kPre = GANNS_LB_PRELOAD != 0 && SPEC;
+    uint64_t worst_pre = kKeyInf;
+    uint32_t probe[3] = {0u, 0u, 0u};
+    if constexpr (kPre) {
+      worst_pre = cnt == l ? unflag(sN[l - 1]) : kKeyInf;
+      if (cnt > 3) {
+        const uint32_t* sNd0 = reinterpret_cast<const uint32_t*>(sN) + 1;
+        const int q0 = cnt >> 2;
+#pragma unroll
+        for (int i = 0; i < 3; ++i) probe[i] = sNd0[2 * ((i + 1) * q0)];
+      }
+    }
     // (3) bulk distance computation
 #pragma unroll
     for (int t = 0; t < TPL; ++t) dist.explore_hint(g, u[t], lane, ws);
@@ -988,7 +1010,7 @@ __device__ int warp_search_with(const GraphView& g, DIST& dist, int32_t entry, i
     GANNS_PROF_MARK(kProfDistance);
     // (4) lazy check (R-C1): drop entries already in N; entries that
     // cannot enter N (>= its l-th key while N is full) are dropped as well.
-    const uint64_t worst = cnt == l ? unflag(sN[l - 1]) : kKeyInf;
+    const uint64_t worst = kPre ? worst_pre : cnt == l ? unflag(sN[l - 1]) : kKeyInf;
 #if GANNS_SKIP_LB
     if (cnt == l) {
       unsigned below = 0;
@@ -1018,6 +1040,12 @@ __device__ int warp_search_with(const GraphView& g, DIST& dist, int32_t entry, i
       const uint64_t kt = key[t];
       const uint32_t kd = uint32_t(kt >> 32);
       int base = 0, len = cnt;   // invariant: lower_bound in [base, base + len]
+      if (kPre && len > 3) {   // the first step on the preloaded probes
+        const int q = len >> 2;
+        const int c = (probe[0] < kd ? 1 : 0) + (probe[1] < kd ? 1 : 0) + (probe[2] < kd ? 1 : 0);
+        base += c * q;
+        len = c < 3 ? q : len - 3 * q;
+      }
       while (len > 3) {
         const int q = len >> 2;
         const int c = (sNd[2 * (base + q)] < kd ? 1 : 0) + (sNd[2 * (base + 2 * q)] < kd ? 1 : 0) +
