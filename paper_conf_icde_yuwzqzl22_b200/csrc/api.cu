@@ -745,9 +745,11 @@ void ganns_hnsw_free(ganns_hnsw* h) {
   int cur = 0;
   cudaGetDevice(&cur);
   cudaSetDevice(h->device);
-  for (auto* p : h->upper) cudaFree(p);
-  cudaFree(h->perm);
-  cudaFree(h->Xp);
+  // like ganns_graph_free: wait for the device, return the index memory to the pool
+  cudaDeviceSynchronize();
+  for (auto* p : h->upper) pool_free(p, nullptr);
+  pool_free(h->perm, nullptr);
+  pool_free(h->Xp, nullptr);
   cudaSetDevice(cur);
   ganns_graph_free(h->base);
   delete h;
@@ -803,12 +805,14 @@ int ganns_build_hnsw(const float* points, int64_t n, int d, int metric, int degr
     if (code) ganns_hnsw_free(h);
     return code;
   };
-  if (cudaMalloc(&h->perm, sizeof(int32_t) * n) != cudaSuccess ||
+  // index memory from the stream-ordered pool (as graph rows: cudaMalloc/cudaFree of
+  // index-sized buffers cost variable host time inside the build)
+  if (pool_alloc(reinterpret_cast<void**>(&h->perm), sizeof(int32_t) * n, s) != cudaSuccess ||
       pool_alloc(reinterpret_cast<void**>(&Xfull), sizeof(float) * size_t(n) * d, s) != cudaSuccess ||
       pool_alloc(reinterpret_cast<void**>(&layer0_shuffled), sizeof(int32_t) * size_t(n) * degree,
                  s) != cudaSuccess)
     return cleanup(fail(GANNS_ENOMEM, "cudaMalloc(hnsw scratch)"));
-  cudaError_t e = cudaMemcpy(h->perm, perm.data(), sizeof(int32_t) * n, cudaMemcpyHostToDevice);
+  cudaError_t e = cudaMemcpyAsync(h->perm, perm.data(), sizeof(int32_t) * n, cudaMemcpyHostToDevice, s);
   if (e == cudaSuccess) e = launch_gather_rows(points, h->perm, n, d, Xfull, s);
   if (e != cudaSuccess) return cleanup(cuda_fail(e, "hnsw permute"));
   // (2) layers top-down, each Algorithm 2 on its prefix
@@ -817,7 +821,8 @@ int ganns_build_hnsw(const float* points, int64_t n, int d, int metric, int degr
   for (int j = top; j >= 0; --j) {
     int32_t* dst = layer0_shuffled;
     if (j >= 1) {
-      if (cudaMalloc(&h->upper[j], sizeof(int32_t) * size_t(layer_n[j]) * degree) != cudaSuccess)
+      if (pool_alloc(reinterpret_cast<void**>(&h->upper[j]), sizeof(int32_t) * size_t(layer_n[j]) * degree,
+                     s) != cudaSuccess)
         return cleanup(fail(GANNS_ENOMEM, "cudaMalloc(hnsw layer)"));
       dst = h->upper[j];
     }
@@ -855,7 +860,8 @@ int ganns_build_hnsw(const float* points, int64_t n, int d, int metric, int degr
   h->base = base;
   e = launch_relabel(layer0_shuffled, h->perm, n, degree, base->nbr, s);
   if (e == cudaSuccess && top >= 1) {
-    if (cudaMalloc(&h->Xp, sizeof(float) * size_t(layer_n[1]) * d) != cudaSuccess)
+    if (pool_alloc(reinterpret_cast<void**>(&h->Xp), sizeof(float) * size_t(layer_n[1]) * d, s) !=
+        cudaSuccess)
       return cleanup(fail(GANNS_ENOMEM, "cudaMalloc(hnsw upper rows)"));
     e = cudaMemcpyAsync(h->Xp, Xfull, sizeof(float) * size_t(layer_n[1]) * d,
                         cudaMemcpyDeviceToDevice, s);
